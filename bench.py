@@ -1,0 +1,351 @@
+#!/usr/bin/env python3
+"""bench.py -- BASELINE.json's metric on its headline single-GPU workload.
+
+Metric: reduced elements/s (and % of B200 HBM peak) at N GPUs vs the CPU oracle.
+Workload (N=1, BASELINE.json configs[1], "cfg2"): 1-D whole-array sum of 2^30
+fp32 elements U[0,1), reduction at gang+worker+vector.  One step = one
+xr_reduce call (the whole hot path: plan, private partials, warp / CTA / last-
+CTA combine, init merge).  N>1 (torchrun): each rank owns its own 2^30-element
+gang slice of a N*2^30 array (weak scaling) and one step = xr_reduce_sharded
+(local kernel + one 4-byte NCCL allreduce over NVLink).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+                  [--workload fp32-sum|fp32-max|fp32-min|int64-sum|int64-max|int64-min]
+
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "reduced elements/s and % of B200 HBM peak (ncu) at 1/2/4/8 GPUs vs CPU oracle"
+WORKLOADS = {
+    # name: (op, dtype, recipe, bytes/elem)
+    "fp32-sum": ("+", "fp32", "u01", 4),
+    "fp32-max": ("max", "fp32", "maxmin", 4),
+    "fp32-min": ("min", "fp32", "maxmin", 4),
+    "int64-sum": ("+", "int64", "ints", 8),
+    "int64-max": ("max", "int64", "maxmin", 8),
+    "int64-min": ("min", "int64", "maxmin", 8),
+}
+DTYPE_TAG = {"fp32": "f32", "fp64": "f64", "int32": "i32", "int64": "i64"}
+N_PER_GPU = 1 << 30
+FALLBACK_HBM_GBS = 6650.0
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="xreduce", choices=["xreduce", "reference"])
+    ap.add_argument("--workload", default="fp32-sum", choices=sorted(WORKLOADS))
+    ap.add_argument("--elements", type=int, default=N_PER_GPU, help="elements per GPU")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    return ap.parse_args()
+
+
+def dist_env():
+    return (int(os.environ.get("RANK", "0")), int(os.environ.get("WORLD_SIZE", "1")),
+            int(os.environ.get("LOCAL_RANK", "0")))
+
+
+def make_input(wl, n, start, total):
+    import datagen
+    from datagen import recipes
+    op, dtype, kind, _ = WORKLOADS[wl]
+    seed = datagen.case_seed(2, {"+": 0, "max": 2, "min": 3}[op], {"fp32": 2, "int64": 1}[dtype], 7)
+    if kind == "ints":  # int64 sum: U_int[-2^31, 2^31)
+        return datagen.uniform_int(seed, n, -(2**31), 2**31 - 1, np.int64, start)
+    return recipes.make(kind, (total, 1, 1), 7, dtype, seed, start=start, n=n)
+
+
+def workload_desc(wl, n, world):
+    op, dtype, kind, _ = WORKLOADS[wl]
+    return {
+        "workload": f"cfg2: 1-D whole-array '{op}' over {n} {dtype} elements per GPU ({kind}), "
+                    f"level_mask gang+worker+vector" + (f", gang-sharded over {world} GPUs + NCCL allreduce"
+                                                       if world > 1 else ""),
+        "nest_dims_per_gpu": [n, 1, 1],
+        "level_mask": "gwv",
+        "op": op,
+        "elements_per_gpu": n,
+        "l2": "input per GPU (%.1f GiB) is larger than L2 (126 MB): no flush needed" % (
+            n * WORKLOADS[wl][3] / 2**30),
+        "parallelism": f"gang-sharded x{world}" if world > 1 else "single GPU",
+    }
+
+
+# --------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,utilization.gpu,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "50"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        try:
+            out, _ = self.p.communicate(timeout=5)
+        except Exception:
+            self.p.kill()
+            out = ""
+        rows = []
+        for line in out.strip().splitlines():
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) >= 8:
+                rows.append(parts)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no samples"], "samples": 0}
+        loaded = [r for r in rows if r[2].isdigit() and int(r[2]) > 0] or rows
+        sm = [int(r[0]) for r in loaded if r[0].isdigit()]
+        mx = [int(r[1]) for r in rows if r[1].isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in loaded for k in range(4) if r[4 + k].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(loaded)}
+
+
+def peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic(wl):
+    """dram bytes per launch of the dominant kernel from the committed ncu capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(wl)
+    except Exception:
+        return None
+
+
+# --------------------------------------------------------------------- CPU oracle legs
+def oracle_rate(wl, x_sample: np.ndarray, seconds: float):
+    """The oracle as it stands, single-threaded, on a bounded sample."""
+    import oracle
+    op, dtype, _, _ = WORKLOADS[wl]
+    n = x_sample.size
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        oracle.reduce(op, dtype, (n, 1, 1), "gwv", x_sample)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            break
+    return reps * n / el, reps, el
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    wl = args.workload
+    n = args.elements
+    sample_n = min(n, 1 << 26)
+    x = make_input(wl, sample_n, 0, n)
+    per_step = []
+    for i in range(args.warmup + args.steps):
+        rate, reps, el = oracle_rate(wl, x, 0.0)
+        if i >= args.warmup:
+            per_step.append(el)
+    t = sum(per_step)
+    value = args.steps * sample_n / t
+    line = {
+        "metric": METRIC, "value": value, "unit": "elements/s", "n_gpus": args.gpus, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": DTYPE_TAG[WORKLOADS[wl][1]],
+        "data": "synthetic (seeded splitmix64 generator, datagen/)", "impl": "reference",
+        "config": workload_desc(wl, n, args.gpus),
+        "cpu_baseline": {"value": value, "unit": "elements/s", "cores": 1, "kind": "oracle",
+                         "sample": f"first {sample_n} elements of the workload per step (plain C oracle, 1 thread)"},
+        "e2e": {"value": value, "unit": "elements/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# --------------------------------------------------------------------- GPU arm
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_xutycc14_b200 as xr
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    wl = args.workload
+    op, dtype, kind, esz = WORKLOADS[wl]
+    n = args.elements
+    total = n * world
+    tdt = {"fp32": torch.float32, "int64": torch.int64}[dtype]
+
+    # inputs: seeded host generation of this rank's gang slice, pinned, then resident in HBM
+    host = torch.from_numpy(make_input(wl, n, rank * n, total)).pin_memory()
+    x = host.to("cuda", non_blocking=False)
+    out = torch.zeros(1, dtype=tdt, device="cuda")
+    stream = torch.cuda.current_stream()
+    sh = stream.cuda_stream
+    comm = xr.Comm() if world > 1 else None
+
+    def step():
+        if comm is None:
+            st = xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), sh)
+        else:
+            st = xr._lib.xr_reduce_sharded(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)), xr.mask_of("gwv"),
+                                           x.data_ptr(), out.data_ptr(), comm.handle, sh)
+        if st != 0:
+            raise xr.XReduceError(st, "bench step")
+
+    for _ in range(max(args.warmup, 3)):
+        step()
+    torch.cuda.synchronize()
+
+    clocks = ClockSampler(local)
+    clocks.start()
+    time.sleep(0.3)  # let the sampler attach
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches0 = xr.xr_launch_count()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for i in range(args.steps):
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches = xr.xr_launch_count() - launches0
+    ck = clocks.stop()
+    total_ms = t_start.elapsed_time(t_end)
+    per = [a.elapsed_time(b) for a, b in ev]
+    if world > 1:
+        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total_ms = float(t.item())
+    ms_step = total_ms / args.steps
+    value = total * args.steps / (total_ms / 1e3)
+
+    # kernel-only duration: at N=1 the step IS the one reduction kernel
+    kern_ms = statistics.mean(per)
+    peak, peak_src = peak_hbm()
+    alg_bytes = n * esz + esz  # read every input element once + write one output
+    achieved = alg_bytes / (kern_ms / 1e3) / 1e9
+    traffic = ncu_traffic(wl)
+
+    # e2e through the C ABI with HOST buffers (H2D of the step's input + D2H of the result)
+    e2e = None
+    if args.e2e_steps > 0:
+        out_h = np.zeros(1, dtype={"fp32": np.float32, "int64": np.int64}[dtype])
+        hp = host.data_ptr()
+        if world == 1:
+            xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)  # warm staging
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            for _ in range(args.e2e_steps):
+                st = xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)
+                assert st == 0
+            el = time.perf_counter() - t0
+        else:
+            dev = torch.empty_like(x)
+            outd = torch.zeros(1, dtype=tdt, device="cuda")
+            dist.barrier()
+            t0 = time.perf_counter()
+            for _ in range(args.e2e_steps):
+                dev.copy_(host, non_blocking=True)
+                st = xr._lib.xr_reduce_sharded(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)), xr.mask_of("gwv"),
+                                               dev.data_ptr(), outd.data_ptr(), comm.handle, sh)
+                assert st == 0
+                outd.cpu()
+            torch.cuda.synchronize()
+            el = time.perf_counter() - t0
+            t = torch.tensor([el], dtype=torch.float64, device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            el = float(t.item())
+        e2e = {"value": total * args.e2e_steps / el, "unit": "elements/s",
+               "h2d_bytes_per_step": n * esz, "d2h_bytes_per_step": esz, "steps": args.e2e_steps,
+               "api": "xr_reduce_host (C ABI, pinned host input)" if world == 1 else
+                      "pinned H2D + xr_reduce_sharded + D2H"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        sample_n = min(n, 1 << 26)
+        rate, reps, el = oracle_rate(wl, host.numpy()[:sample_n], args.cpu_seconds)
+        cpu = {"value": rate, "unit": "elements/s", "cores": 1, "kind": "oracle",
+               "sample": f"{reps} x oracle over the first {sample_n} elements ({el:.1f} s, 1 thread)"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": DTYPE_TAG[dtype],
+            "data": "synthetic (seeded splitmix64 generator, datagen/)",
+            "config": workload_desc(wl, n, world),
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "peak_source": peak_src,
+                         "kernel": "seg_kernel<W=CTA> (xr_reduce R-shape)",
+                         "algorithmic_bytes_per_launch": alg_bytes,
+                         "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)},
+            "hbm_frac_of_peak": achieved / peak,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": ck,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.close()
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_gpu(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

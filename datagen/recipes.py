@@ -24,6 +24,9 @@ Recipe names (``kind``):
   land      non-zero with zeros (incl. -0.0) at rate 0.7/L (P7)
   lor       zeros (+-0.0) with non-zeros at rate 0.7/L (P7)
   specials  U[-1,1) with NaN, +-inf, +-0, subnormals planted (floats only)
+  mulspecials  the ``mul`` recipe (exact power-of-two products) with NaN, +-inf,
+            +-0 planted -- products of specials without intermediate
+            under/overflow, the only regime where products are order independent
 """
 from __future__ import annotations
 
@@ -146,6 +149,16 @@ def make(kind: str, dims, mask: int, dtype, seed: int, start: int = 0, n: int | 
         table = [np.nan, np.inf, -np.inf, 0.0, -0.0, tiny, -tiny]
         plant = _rate(_sub(seed, 12), n, start, 3.0, L)
         for k, v in enumerate(table):
+            x[plant & (pick == k)] = v
+        return x
+    if kind == "mulspecials":
+        if isint:
+            raise ValueError("mulspecials is a floating-point recipe")
+        x = make("mul", dims, mask, dtype, seed, start, n)
+        h = hashes(_sub(seed, 13), n, start)
+        pick = (h % np.uint64(8)).astype(np.int64)
+        plant = _rate(_sub(seed, 14), n, start, 2.0, L)
+        for k, v in enumerate([np.nan, np.inf, -np.inf, 0.0, -0.0]):
             x[plant & (pick == k)] = v
         return x
     raise ValueError(f"unknown recipe {kind!r}")

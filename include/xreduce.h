@@ -1,0 +1,244 @@
+/*
+ * include/xreduce.h -- C ABI of xreduce, the B200-native (sm_100a) hot path of
+ * Xu et al., "Reduction Operations in Parallel Loops for GPGPUs" (PMAM'14).
+ *
+ * Citations are PAPER.md:1 character offsets (@N; the extracted paper is one
+ * line) with the section they fall in.  See DESIGN.md for the readings C1-C23
+ * adopted where the paper is silent or garbled.
+ *
+ * The problem (PAPER.md @4654-4854, section 1; again @13077-13277, section 3):
+ * "a binary associative operator to operate an input array and generate a
+ * single output value", placed on any of the three loop levels of a nest
+ * (gang = outer k, worker = middle j, vector = inner i; @9947-10334, 2.2) or
+ * on several of them (RMP, @26751-27253, 3.2).  Levels that are not reduced
+ * "execute in parallel" (@44766, Table 2 caption) and yield one result per
+ * iteration (Fig 4: temp[k][j][0] = i_sum, @17176).  The variable's original
+ * value is combined after the reduction (@21488-21990, 3.1.1).
+ *
+ * Conventions (every entry point):
+ *  - Return an xr_status; 0 = success.  No C++ exception crosses the ABI.
+ *  - Argument validation runs BEFORE any CUDA call, so invalid calls return
+ *    XR_ERR_INVALID / XR_ERR_UNSUPPORTED on machines without a GPU.
+ *  - Device calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy
+ *    default stream); results are valid after the stream synchronises.  No
+ *    host synchronisation happens inside xr_reduce except when the library's
+ *    workspace must grow (first calls only; see xr_reserve).
+ *  - Thread-safe across host threads.  Concurrent calls on DIFFERENT streams
+ *    use different workspaces.
+ */
+#ifndef XREDUCE_H
+#define XREDUCE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* Compatible with cudaStream_t (both are `struct CUstream_st *`). */
+typedef struct CUstream_st* xr_stream_t;
+
+/* Operators (reading C1: the OpenACC C set; the paper evaluates + and *
+ * (@37852-37985) and max (@37985, Fig 13a) and claims "all reduction
+ * operator types" (@6300-6414)). */
+typedef enum {
+  XR_OP_ADD = 0,  /* +   identity 0 (+0.0 for fp)                           */
+  XR_OP_MUL = 1,  /* *   identity 1                                          */
+  XR_OP_MAX = 2,  /* max identity lowest (INT_MIN / -inf); fp: NaN operands
+                     ignored, -0 < +0 (reading C7)                           */
+  XR_OP_MIN = 3,  /* min identity highest (INT_MAX / +inf); same fp rule     */
+  XR_OP_BAND = 4, /* &   identity ~0        (integers only, reading C3)      */
+  XR_OP_BOR = 5,  /* |   identity 0         (integers only)                  */
+  XR_OP_BXOR = 6, /* ^   identity 0         (integers only)                  */
+  XR_OP_LAND = 7, /* &&  identity 1; truth = (x != 0); result 0/1 in dtype (C8) */
+  XR_OP_LOR = 8   /* ||  identity 0; result 0/1 in dtype                     */
+} xr_op;
+
+/* Operand types: Table 2's int / float / double (@45106-45160) plus int64
+ * (reading C2).  The output has the input's type.  Integer + and * wrap
+ * modulo 2^32 / 2^64 (reading C6). */
+typedef enum { XR_INT32 = 0, XR_INT64 = 1, XR_FP32 = 2, XR_FP64 = 3 } xr_dtype;
+
+/* Level bits of `level_mask`.  nest_dims = {n0, n1, n2} describes the
+ * row-major array in[k][j][i] with k < n0 (gang, outermost), j < n1 (worker),
+ * i < n2 (vector, contiguous) -- the paper's mapping "k loop ... across all
+ * gangs, j ... across all workers ..., i ... across all vector threads"
+ * (@10531-11313, Fig 2/3). */
+#define XR_GANG 0x1u
+#define XR_WORKER 0x2u
+#define XR_VECTOR 0x4u
+/* out[] holds per-output initial values (the paper's "original value",
+ * @21488-21990); otherwise the initial value is the identity. */
+#define XR_INIT_FROM_OUT 0x100u
+
+typedef enum {
+  XR_OK = 0,
+  XR_ERR_INVALID = 1,     /* bad op/dtype code, mask, dims, pointer, overlap  */
+  XR_ERR_UNSUPPORTED = 2, /* & | ^ on fp32/fp64 (reading C3)                  */
+  XR_ERR_CUDA = 3,        /* a CUDA runtime error (launch, allocation, copy)  */
+  XR_ERR_NCCL = 4,        /* an NCCL error (sharded calls)                    */
+  XR_ERR_NOMEM = 5        /* workspace allocation failed                      */
+} xr_status;
+
+/* ---------------------------------------------------------------- core ---- */
+
+/* xr_reduce -- out[o] = init[o] (+) OP over the reduced levels of in.
+ *
+ *   op, dtype   : xr_op, xr_dtype.  30 legal pairs: + * max min && || on all
+ *                 four types, & | ^ on int32/int64 (else XR_ERR_UNSUPPORTED).
+ *   nest_dims   : host pointer to 3 extents n0, n1, n2 >= 0 whose product
+ *                 fits in int64 (else XR_ERR_INVALID).
+ *   level_mask  : OR of XR_GANG / XR_WORKER / XR_VECTOR (at least one),
+ *                 optionally | XR_INIT_FROM_OUT; other bits -> XR_ERR_INVALID.
+ *                 Every combination is defined, including gang+vector without
+ *                 worker (reading C13; the paper says it "cannot span across
+ *                 gang & vector without going through the worker", @29561).
+ *   in          : DEVICE pointer, n0*n1*n2 elements, dtype-aligned (4 or 8 B;
+ *                 16 B alignment is NOT required).  Caller-owned, read only.
+ *   out         : DEVICE pointer, xr_out_count elements, compact row-major over
+ *                 the kept levels in (k, j, i) order (reading C11).  Must not
+ *                 overlap in (XR_ERR_INVALID).  Read first when
+ *                 XR_INIT_FROM_OUT is set, then overwritten.
+ *   stream      : launch stream.
+ * A kept extent of 0 gives an empty output (no-op).  A reduced extent of 0
+ * gives out = init (reading C17).  Null pointers with non-empty work ->
+ * XR_ERR_INVALID.  One kernel launch per call (single pass: per-CTA partials
+ * combined by the last CTA to finish, no second launch). */
+int xr_reduce(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+              const void* in, void* out, xr_stream_t stream);
+
+/* Number of outputs: the product of the kept extents (1 if all reduced). */
+int xr_out_count(const int64_t nest_dims[3], unsigned level_mask, int64_t* count);
+
+/* Static string for a status code (never NULL). */
+const char* xr_strerror(int status);
+
+/* Same as xr_reduce but with HOST buffers: copies in (host, pinned or
+ * pageable) to a library-owned device staging buffer in chunks along the gang
+ * level, overlapping the copy of chunk c+1 with the reduction of chunk c, and
+ * copies the result back into out (host).  Synchronous: returns after out is
+ * written.  `stream` orders the work; NULL uses the legacy stream. */
+int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+                   const void* in_host, void* out_host, xr_stream_t stream);
+
+/* ------------------------------------------------------------ planning ---- */
+
+/* Canonical shapes after dropping extent-1 levels and merging adjacent levels
+ * of the same status.  R = reduced run, K = kept run. */
+typedef enum {
+  XR_SHAPE_NONE = 0,  /* empty output: nothing to do                        */
+  XR_SHAPE_FILL = 1,  /* a reduced extent is 0: out = init                  */
+  XR_SHAPE_IDENT = 2, /* "K": every reduced extent is 1: out = init (+) in  */
+  XR_SHAPE_R = 3,     /* whole-nest scalar                                   */
+  XR_SHAPE_KR = 4,    /* keep outer, reduce contiguous inner (rows)          */
+  XR_SHAPE_RK = 5,    /* reduce outer, keep contiguous inner (columns)       */
+  XR_SHAPE_KRK = 6,   /* batched columns                                     */
+  XR_SHAPE_RKR = 7    /* keep the middle, reduce outer and inner             */
+} xr_shape;
+
+typedef struct {
+  int shape;            /* xr_shape                                          */
+  int kernel;           /* 0 none, 1 fill, 2 ident, 3 seg, 4 col             */
+  int64_t cdims[3];     /* canonical extents (shape-dependent, rest 0)       */
+  int64_t out_count;
+  int group;            /* seg: lanes per group (8, 32 or the CTA size)      */
+  int vec;              /* elements per 16-byte load (col: 1 if unaligned)    */
+  int64_t splits;       /* partial units per output (1 = no gang-tier combine) */
+  int64_t units;        /* total work units                                  */
+  int64_t grid;         /* CTAs launched                                     */
+  int block;            /* threads per CTA                                   */
+  int64_t ws_bytes;     /* workspace bytes (partials)                        */
+  int64_t tickets;      /* last-CTA tickets                                  */
+} xr_plan_info;
+
+/* Host-only: the plan xr_reduce would use on a device with `num_sms` SMs.
+ * `in_addr` is the input address (only its alignment matters).  No CUDA. */
+int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+                     uint64_t in_addr, int num_sms, xr_plan_info* info);
+
+/* Pre-grow the workspace of (current device, stream) for the given call so
+ * that later calls never allocate (e.g. before CUDA-graph capture). */
+int xr_reserve(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+               xr_stream_t stream);
+
+/* Release every workspace and staging buffer (synchronises the device). */
+int xr_shutdown(void);
+
+/* Number of kernels this library has launched in this process. */
+int64_t xr_launch_count(void);
+
+/* --------------------------------------------------------- heat (cfg 4) ---- */
+
+/* One fused Jacobi sweep + max-residual reduction of the 2-D heat equation
+ * (Fig 13(a) @43561-44280, section 4 @39322-41386; reading C14):
+ *   T2[j][i] = 0.25*((T1[j-1][i] + T1[j+1][i]) + (T1[j][i-1] + T1[j][i+1]))
+ * for 1 <= j < nj-1, 1 <= i < ni-1 (no FMA contraction), and
+ *   *residual = max(0, max |T2 - T1|)   (gang+worker+vector max, one launch).
+ * T1, T2: DEVICE nj x ni row-major fp64; T2's boundary must already hold the
+ * boundary values (it is never written).  residual: DEVICE pointer to 1 fp64. */
+int xr_heat_step(int64_t nj, int64_t ni, const double* T1, double* T2, double* residual,
+                 xr_stream_t stream);
+
+/* iters sweeps, swapping T1/T2; residuals[it] (DEVICE, iters fp64).  The
+ * newest field is in T1 when iters is even, in T2 when odd. */
+int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,
+                double* residuals, xr_stream_t stream);
+
+/* ------------------------------------------------- multi-GPU (gang shards) */
+
+/* Sharding along the gang level: rank r owns the contiguous
+ * gang slice [r*n0_local, (r+1)*n0_local); every rank passes the same
+ * local_dims.  After the call, out on EVERY rank holds the GLOBAL result:
+ *   G in mask : xr_out_count(local_dims) elements (partials combined);
+ *   G not in  : nranks * xr_out_count(local_dims) elements, rank-major
+ *               (= global row-major, because gang is outermost).
+ * XR_INIT_FROM_OUT with G in mask merges rank 0's init exactly once; with G
+ * not in mask each rank merges the init of its own segment. */
+typedef enum {
+  XR_COLL_NONE = 0,
+  XR_COLL_ALLREDUCE = 1,        /* ncclSum/Prod/Max/Min (&& -> Min, || -> Max on 0/1) */
+  XR_COLL_ALLGATHER_COMBINE = 2,/* & | ^ : gather partials, fixed rank-order combine  */
+  XR_COLL_ALLGATHER = 3         /* gang kept: gather disjoint output segments          */
+} xr_collective;
+
+typedef struct {
+  int collective;        /* xr_collective                                    */
+  int nccl_op;           /* ncclRedOp_t for XR_COLL_ALLREDUCE, else -1        */
+  int merge_init;        /* 1 if this rank merges the caller's init locally   */
+  int local_init_from_out; /* 1 if the local reduction reads out as init      */
+  int64_t local_count;   /* outputs of the local reduction                    */
+  int64_t global_count;  /* outputs after the exchange                         */
+  int64_t out_offset;    /* where this rank's local result lands in out        */
+  int64_t gang_offset;   /* first global gang index owned by this rank         */
+} xr_shard_info;
+
+/* Host-only: the exchange xr_reduce_sharded performs for this rank. */
+int xr_shard_plan(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                  int nranks, int rank, xr_shard_info* info);
+
+typedef struct xr_comm_s* xr_comm_t;
+
+/* NCCL unique id (128 bytes) on rank 0; broadcast it out of band
+ * (torch.distributed in the Python binding). */
+int xr_comm_get_unique_id(void* id128);
+/* One communicator per process/GPU (device = CUDA ordinal used by this rank). */
+int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int device);
+int xr_comm_destroy(xr_comm_t comm);
+
+/* Local xr_reduce on this rank's gang slice + ONE collective on `stream`. */
+int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                      const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream);
+
+/* Single-device simulation of the sharded protocol (testing without NCCL):
+ * shards[r] (DEVICE) holds rank r's slice; runs the nranks local reductions
+ * and the same exchange semantics with device copies + the same fixed-order
+ * combine kernel.  out as for rank 0 of xr_reduce_sharded. */
+int xr_reduce_sharded_sim(int op, int dtype, const int64_t local_dims[3],
+                          unsigned level_mask, const void* const* shards, int nranks,
+                          void* out, xr_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* XREDUCE_H */

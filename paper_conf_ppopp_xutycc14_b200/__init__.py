@@ -1,0 +1,292 @@
+"""xreduce -- B200-native (sm_100a) parallel reductions over 1-3 level loop nests.
+
+Thin ctypes binding over ``libxreduce.so`` (include/xreduce.h).  Argument
+marshalling only: every step of the reduction runs in the library's CUDA
+kernels.  PyTorch is used for device memory, streams and process groups.
+There is NO CPU fallback: if the shared library is missing this import fails
+loudly (build it with ``python -m paper_conf_ppopp_xutycc14_b200._build`` or
+``__graft_entry__.build()``).
+
+Paper: Xu, Tian, Yan, Chandrasekaran, Chapman, "Reduction Operations in
+Parallel Loops for GPGPUs", PMAM'14; see DESIGN.md.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libxreduce.so")
+if not os.path.exists(LIB_PATH):
+    raise ImportError(
+        f"xreduce: {LIB_PATH} is missing -- build the CUDA library first "
+        "(python -m paper_conf_ppopp_xutycc14_b200._build); there is no CPU fallback")
+_lib = ctypes.CDLL(LIB_PATH)
+
+# ---- codes (include/xreduce.h)
+OP_ADD, OP_MUL, OP_MAX, OP_MIN, OP_BAND, OP_BOR, OP_BXOR, OP_LAND, OP_LOR = range(9)
+INT32, INT64, FP32, FP64 = range(4)
+GANG, WORKER, VECTOR, INIT_FROM_OUT = 0x1, 0x2, 0x4, 0x100
+OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL, ERR_NOMEM = range(6)
+SHAPES = {0: "none", 1: "fill", 2: "ident", 3: "R", 4: "KR", 5: "RK", 6: "KRK", 7: "RKR"}
+KERNELS = {0: "none", 1: "fill", 2: "ident", 3: "seg", 4: "col"}
+COLL_NONE, COLL_ALLREDUCE, COLL_ALLGATHER_COMBINE, COLL_ALLGATHER = range(4)
+
+OPS = {"+": OP_ADD, "*": OP_MUL, "max": OP_MAX, "min": OP_MIN, "&": OP_BAND, "|": OP_BOR,
+       "^": OP_BXOR, "&&": OP_LAND, "||": OP_LOR}
+DTYPES = {"int32": INT32, "int64": INT64, "fp32": FP32, "fp64": FP64}
+
+
+class XReduceError(RuntimeError):
+    def __init__(self, status: int, where: str = ""):
+        msg = _lib.xr_strerror(status).decode()
+        super().__init__(f"{where}: {msg}" if where else msg)
+        self.status = status
+
+
+class PlanInfo(ctypes.Structure):
+    _fields_ = [("shape", ctypes.c_int), ("kernel", ctypes.c_int),
+                ("cdims", ctypes.c_int64 * 3), ("out_count", ctypes.c_int64),
+                ("group", ctypes.c_int), ("vec", ctypes.c_int), ("splits", ctypes.c_int64),
+                ("units", ctypes.c_int64), ("grid", ctypes.c_int64), ("block", ctypes.c_int),
+                ("ws_bytes", ctypes.c_int64), ("tickets", ctypes.c_int64)]
+
+    def as_dict(self):
+        d = {f: getattr(self, f) for f, _ in self._fields_}
+        d["cdims"] = list(self.cdims)
+        d["shape"] = SHAPES[self.shape]
+        d["kernel"] = KERNELS[self.kernel]
+        return d
+
+
+class ShardInfo(ctypes.Structure):
+    _fields_ = [("collective", ctypes.c_int), ("nccl_op", ctypes.c_int),
+                ("merge_init", ctypes.c_int), ("local_init_from_out", ctypes.c_int),
+                ("local_count", ctypes.c_int64), ("global_count", ctypes.c_int64),
+                ("out_offset", ctypes.c_int64), ("gang_offset", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+_i64p = ctypes.POINTER(ctypes.c_int64)
+_vp = ctypes.c_void_p
+_c = ctypes.c_int
+_u = ctypes.c_uint
+
+_SIGS = {
+    "xr_reduce": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp]),
+    "xr_out_count": (_c, [_i64p, _u, _i64p]),
+    "xr_strerror": (ctypes.c_char_p, [_c]),
+    "xr_reduce_host": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp]),
+    "xr_plan_describe": (_c, [_c, _c, _i64p, _u, ctypes.c_uint64, _c, ctypes.POINTER(PlanInfo)]),
+    "xr_reserve": (_c, [_c, _c, _i64p, _u, _vp]),
+    "xr_shutdown": (_c, []),
+    "xr_launch_count": (ctypes.c_int64, []),
+    "xr_heat_step": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp]),
+    "xr_heat_run": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp]),
+    "xr_shard_plan": (_c, [_c, _c, _i64p, _u, _c, _c, ctypes.POINTER(ShardInfo)]),
+    "xr_comm_get_unique_id": (_c, [_vp]),
+    "xr_comm_init": (_c, [ctypes.POINTER(_vp), _c, _c, _vp, _c]),
+    "xr_comm_destroy": (_c, [_vp]),
+    "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
+    "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
+}
+for _name, (_res, _args) in _SIGS.items():
+    _f = getattr(_lib, _name)
+    _f.restype = _res
+    _f.argtypes = _args
+
+EXPORTED = tuple(_SIGS)
+
+
+def _dims(d):
+    return (ctypes.c_int64 * 3)(*[int(v) for v in d])
+
+
+def _check(st: int, where: str):
+    if st != OK:
+        raise XReduceError(st, where)
+
+
+def mask_of(levels) -> int:
+    """'gwv'-style string (or an int) -> level mask."""
+    if isinstance(levels, int):
+        return levels
+    m = 0
+    for ch in levels.lower():
+        m |= {"g": GANG, "w": WORKER, "v": VECTOR}[ch]
+    return m
+
+
+def _op(op):
+    return OPS[op] if isinstance(op, str) else int(op)
+
+
+def _dt(dt):
+    return DTYPES[dt] if isinstance(dt, str) else int(dt)
+
+
+# ---------------------------------------------------------------- raw C ABI
+def xr_reduce(op, dtype, nest_dims, level_mask, in_ptr: int, out_ptr: int, stream: int = 0) -> int:
+    return _lib.xr_reduce(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask),
+                          in_ptr or None, out_ptr or None, stream or None)
+
+
+def xr_out_count(nest_dims, level_mask) -> int:
+    c = ctypes.c_int64(0)
+    _check(_lib.xr_out_count(_dims(nest_dims), mask_of(level_mask), ctypes.byref(c)), "xr_out_count")
+    return int(c.value)
+
+
+def xr_strerror(status: int) -> str:
+    return _lib.xr_strerror(status).decode()
+
+
+def xr_plan_describe(op, dtype, nest_dims, level_mask, in_addr: int = 0, num_sms: int = 148) -> dict:
+    info = PlanInfo()
+    _check(_lib.xr_plan_describe(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask),
+                                 in_addr, num_sms, ctypes.byref(info)), "xr_plan_describe")
+    return info.as_dict()
+
+
+def xr_shard_plan(op, dtype, local_dims, level_mask, nranks: int, rank: int) -> dict:
+    info = ShardInfo()
+    _check(_lib.xr_shard_plan(_op(op), _dt(dtype), _dims(local_dims), mask_of(level_mask),
+                              nranks, rank, ctypes.byref(info)), "xr_shard_plan")
+    return info.as_dict()
+
+
+def xr_reduce_host(op, dtype, nest_dims, level_mask, in_host_ptr: int, out_host_ptr: int,
+                   stream: int = 0) -> int:
+    return _lib.xr_reduce_host(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask),
+                               in_host_ptr or None, out_host_ptr or None, stream or None)
+
+
+def xr_reserve(op, dtype, nest_dims, level_mask, stream: int = 0) -> int:
+    return _lib.xr_reserve(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask), stream or None)
+
+
+def xr_shutdown() -> int:
+    return _lib.xr_shutdown()
+
+
+def xr_launch_count() -> int:
+    return int(_lib.xr_launch_count())
+
+
+def xr_heat_step(nj, ni, t1_ptr, t2_ptr, residual_ptr, stream: int = 0) -> int:
+    return _lib.xr_heat_step(nj, ni, t1_ptr, t2_ptr, residual_ptr, stream or None)
+
+
+def xr_heat_run(nj, ni, iters, t1_ptr, t2_ptr, residuals_ptr, stream: int = 0) -> int:
+    return _lib.xr_heat_run(nj, ni, iters, t1_ptr, t2_ptr, residuals_ptr, stream or None)
+
+
+def xr_reduce_sharded_sim(op, dtype, local_dims, level_mask, shard_ptrs, out_ptr, stream: int = 0) -> int:
+    arr = (_vp * len(shard_ptrs))(*shard_ptrs)
+    return _lib.xr_reduce_sharded_sim(_op(op), _dt(dtype), _dims(local_dims), mask_of(level_mask),
+                                      arr, len(shard_ptrs), out_ptr, stream or None)
+
+
+# ---------------------------------------------------------------- torch-facing helpers
+_TORCH_DT = None
+
+
+def _torch_dtypes():
+    global _TORCH_DT
+    if _TORCH_DT is None:
+        import torch
+        _TORCH_DT = {torch.int32: INT32, torch.int64: INT64, torch.float32: FP32, torch.float64: FP64}
+    return _TORCH_DT
+
+
+def _stream_handle(stream=None) -> int:
+    import torch
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def reduce(x, op="+", levels="gwv", nest=None, out=None, init=None, stream=None):
+    """Reduce CUDA tensor ``x`` (viewed as nest ``(n0, n1, n2)``, default: x.shape
+    padded to 3 dims on the left) over ``levels``; returns the compact output
+    tensor (shape = the kept extents)."""
+    import torch
+    if not x.is_cuda:
+        raise ValueError("xreduce.reduce needs a CUDA tensor (no CPU fallback)")
+    x = x.contiguous()
+    if nest is None:
+        shp = list(x.shape)[-3:]
+        nest = [1] * (3 - len(shp)) + shp
+    nest = [int(v) for v in nest]
+    mask = mask_of(levels)
+    dt = _torch_dtypes()[x.dtype]
+    kept = [nest[d] for d in range(3) if not (mask >> d) & 1]
+    count = xr_out_count(nest, mask)
+    if out is None:
+        out = torch.empty(kept if kept else [1], dtype=x.dtype, device=x.device)
+    if init is not None:
+        out.copy_(torch.as_tensor(init, dtype=x.dtype, device=x.device).reshape(out.shape))
+        mask |= INIT_FROM_OUT
+    assert out.numel() == count and out.is_contiguous()
+    _check(xr_reduce(_op(op), dt, nest, mask, x.data_ptr(), out.data_ptr(), _stream_handle(stream)),
+           "xr_reduce")
+    return out
+
+
+class Comm:
+    """An xreduce NCCL communicator built over a torch.distributed process group
+    (the 128-byte NCCL unique id is broadcast with torch.distributed)."""
+
+    def __init__(self, group=None, device: int | None = None):
+        import torch
+        import torch.distributed as dist
+        self.rank = dist.get_rank(group)
+        self.nranks = dist.get_world_size(group)
+        self.device = torch.cuda.current_device() if device is None else device
+        uid = (ctypes.c_char * 128)()
+        if self.rank == 0:
+            _check(_lib.xr_comm_get_unique_id(ctypes.cast(uid, _vp)), "xr_comm_get_unique_id")
+        obj = [bytes(uid) if self.rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0, group=group)
+        uid = (ctypes.c_char * 128).from_buffer_copy(obj[0])
+        self._h = _vp()
+        _check(_lib.xr_comm_init(ctypes.byref(self._h), self.nranks, self.rank,
+                                 ctypes.cast(uid, _vp), self.device), "xr_comm_init")
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if self._h:
+            _check(_lib.xr_comm_destroy(self._h), "xr_comm_destroy")
+            self._h = _vp()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def reduce_sharded(x_local, comm: Comm, op="+", levels="gwv", nest_local=None, out=None, init=None,
+                   stream=None):
+    """Gang-sharded reduction: every rank passes its contiguous gang slice;
+    returns the GLOBAL result on every rank (include/xreduce.h)."""
+    import torch
+    x_local = x_local.contiguous()
+    if nest_local is None:
+        shp = list(x_local.shape)[-3:]
+        nest_local = [1] * (3 - len(shp)) + shp
+    mask = mask_of(levels)
+    info = xr_shard_plan(op, _torch_dtypes()[x_local.dtype], nest_local, mask, comm.nranks, comm.rank)
+    if out is None:
+        out = torch.empty(max(info["global_count"], 1), dtype=x_local.dtype, device=x_local.device)
+    if init is not None:
+        out.copy_(torch.as_tensor(init, dtype=x_local.dtype, device=out.device).reshape(out.shape))
+        mask |= INIT_FROM_OUT
+    _check(_lib.xr_reduce_sharded(_op(op), _torch_dtypes()[x_local.dtype], _dims(nest_local), mask,
+                                  x_local.data_ptr(), out.data_ptr(), comm.handle,
+                                  _stream_handle(stream)), "xr_reduce_sharded")
+    return out

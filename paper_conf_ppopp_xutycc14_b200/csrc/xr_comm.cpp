@@ -1,0 +1,126 @@
+// xr_comm.cpp -- multi-GPU gang sharding.
+//
+// In the paper, gangs compute independent private partials and only the
+// cross-gang combine needs a global synchronisation, which thread blocks
+// cannot do (PAPER.md @7679, @24887-25280).  Across GPUs the same structure
+// holds: each rank reduces its contiguous gang slice with the single-GPU path
+// (blocking across GPUs; the paper notes blocking and window sliding are
+// equivalent for gang partial reduction, @25998-26464), then ONE collective
+// over NVLink/NVSwitch combines them (xr_shard_plan decides which).
+#include <cstring>
+#include <nccl.h>
+
+#include "../../include/xreduce.h"
+#include "xr_internal.h"
+
+namespace xr {
+int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask, const void* in, void* out,
+                          cudaStream_t s);
+cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+}  // namespace xr
+
+struct xr_comm_s {
+  ncclComm_t nccl = nullptr;
+  int nranks = 0, rank = 0, device = 0;
+  void* scratch = nullptr;  // allgather buffers for & | ^
+  size_t scratch_bytes = 0;
+};
+
+using namespace xr;
+
+static ncclDataType_t nccl_type(int dtype) {
+  switch (dtype) {
+    case XR_INT32: return ncclInt32;
+    case XR_INT64: return ncclInt64;
+    case XR_FP32: return ncclFloat32;
+    default: return ncclFloat64;
+  }
+}
+
+extern "C" {
+
+int xr_comm_get_unique_id(void* id128) {
+  if (!id128) return XR_ERR_INVALID;
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return XR_ERR_NCCL;
+  std::memcpy(id128, &id, sizeof id);
+  return XR_OK;
+}
+
+int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int device) {
+  if (!comm || !id128 || nranks < 1 || rank < 0 || rank >= nranks || device < 0) return XR_ERR_INVALID;
+  if (cudaSetDevice(device) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  ncclUniqueId id;
+  std::memcpy(&id, id128, sizeof id);
+  xr_comm_s* c = new xr_comm_s();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = device;
+  if (ncclCommInitRank(&c->nccl, nranks, id, rank) != ncclSuccess) {
+    delete c;
+    return XR_ERR_NCCL;
+  }
+  *comm = c;
+  return XR_OK;
+}
+
+int xr_comm_destroy(xr_comm_t comm) {
+  if (!comm) return XR_ERR_INVALID;
+  int st = XR_OK;
+  if (comm->scratch) cudaFree(comm->scratch);
+  if (comm->nccl && ncclCommDestroy(comm->nccl) != ncclSuccess) st = XR_ERR_NCCL;
+  delete comm;
+  return st;
+}
+
+int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                      const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream) {
+  if (!comm) return XR_ERR_INVALID;
+  xr_shard_info info;
+  int st = xr_shard_plan(op, dtype, local_dims, level_mask, comm->nranks, comm->rank, &info);
+  if (st) return st;
+  if (info.global_count == 0) return XR_OK;
+  if (!out) return XR_ERR_INVALID;
+  cudaStream_t s = (cudaStream_t)stream;
+  const int size = dtype_size(dtype);
+  const unsigned base = (level_mask & 7u) | (info.local_init_from_out ? XR_INIT_FROM_OUT : 0u);
+  char* mine = (char*)out + info.out_offset * size;
+
+  if (info.collective == XR_COLL_ALLGATHER_COMBINE) {
+    // & | ^: NCCL has no bitwise reduction -> gather partials, fixed-order combine
+    const size_t need = (size_t)(comm->nranks + 1) * info.local_count * size;
+    if (need > comm->scratch_bytes) {
+      if (comm->scratch) { cudaStreamSynchronize(s); cudaFree(comm->scratch); }
+      comm->scratch = nullptr;
+      comm->scratch_bytes = 0;
+      if (cudaMalloc(&comm->scratch, need) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+      comm->scratch_bytes = need;
+    }
+    char* local = (char*)comm->scratch;
+    char* gathered = local + (size_t)info.local_count * size;
+    if (info.local_init_from_out &&
+        cudaMemcpyAsync(local, out, (size_t)info.local_count * size, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+      return XR_ERR_CUDA;
+    if ((st = reduce_device_checked(op, dtype, local_dims, base, in_local, local, s))) return st;
+    if (ncclAllGather(local, gathered, (size_t)info.local_count, nccl_type(dtype), comm->nccl, s) != ncclSuccess)
+      return XR_ERR_NCCL;
+    if (gather_combine(op, dtype, gathered, comm->nranks, info.local_count, out, s) != cudaSuccess)
+      return XR_ERR_CUDA;
+    return XR_OK;
+  }
+
+  if ((st = reduce_device_checked(op, dtype, local_dims, base, in_local, mine, s))) return st;
+  if (comm->nranks == 1) return XR_OK;
+  if (info.collective == XR_COLL_ALLREDUCE) {
+    if (ncclAllReduce(out, out, (size_t)info.global_count, nccl_type(dtype), (ncclRedOp_t)info.nccl_op,
+                      comm->nccl, s) != ncclSuccess)
+      return XR_ERR_NCCL;
+  } else if (info.collective == XR_COLL_ALLGATHER) {
+    // in place: rank r's segment already sits at out + r*local_count
+    if (ncclAllGather(mine, out, (size_t)info.local_count, nccl_type(dtype), comm->nccl, s) != ncclSuccess)
+      return XR_ERR_NCCL;
+  }
+  return XR_OK;
+}
+
+}  // extern "C"

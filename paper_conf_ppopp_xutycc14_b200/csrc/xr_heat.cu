@@ -1,0 +1,169 @@
+// xr_heat.cu -- config 4: the paper's 2-D heat equation application with its
+// per-iteration max-residual reduction (section 4 @39322-41386,
+// Fig 13(a) @43561-44280), fused into ONE kernel per sweep:
+//
+//   T2[j][i] = 0.25*((T1[j-1][i] + T1[j+1][i]) + (T1[j][i-1] + T1[j][i+1]))
+//   residual = max(0, max_{j,i} |T1[j][i] - T2[j][i]|)       (reading C14)
+//
+// The paper runs the update and then a separate gang(+vector) max reduction
+// that re-reads temp1/temp2 and copies `error` to the host every iteration
+// (@40016-40410); fusing the residual into the sweep makes it free: 16 B per
+// point per iteration (read T1 once from HBM, write T2 once; neighbours come
+// from registers, shuffles and L1), and the reduction reuses the warp / CTA /
+// last-CTA tiers of xr_ops.cuh.  Arithmetic uses __dadd_rn/__dmul_rn so no FMA
+// contraction can occur (the paper disables FMA, @35389-35893), which makes
+// the result bit-identical to the oracle.
+#include "../../include/xreduce.h"
+#include "xr_internal.h"
+#include "xr_ops.cuh"
+
+namespace xr {
+
+int heat_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets);
+
+constexpr int kHeatRows = 32;  // rows marched per warp
+
+struct HeatArgs {
+  const double* T1;
+  double* T2;
+  double* residual;
+  double* partials;
+  unsigned* tickets;
+  int64_t nj, ni;
+  int64_t ntiles;  // CTAs in the grid
+};
+
+__device__ __forceinline__ double stencil(double up, double down, double left, double right) {
+  return __dmul_rn(0.25, __dadd_rn(__dadd_rn(up, down), __dadd_rn(left, right)));
+}
+
+__device__ __forceinline__ double ld_row(const double* p) { return __ldg(p); }
+
+// VEC = columns per lane (2: 16-B loads, needs ni even and 16-B aligned rows).
+template <int VEC>
+__global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
+  using O = Op<OP_MAX, double>;
+  constexpr int NW = kBlock / 32;
+  constexpr int STRIP = 32 * VEC;
+  __shared__ double smem[32];
+  __shared__ int s_last;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t c0 = ((int64_t)blockIdx.x * NW + warp) * STRIP;  // first column of my strip
+  const int64_t col = c0 + (int64_t)lane * VEC;                   // my first column
+  const int64_t j0 = 1 + (int64_t)blockIdx.y * kHeatRows;
+  const int64_t j1 = min(j0 + kHeatRows, a.nj - 1);
+  const int64_t ni = a.ni;
+  double err = 0.0;  // |d| >= 0, and the residual's initial value is 0 (C14)
+
+  if (j0 < j1 && c0 < ni) {
+    const bool have = col < ni;
+    auto load = [&](int64_t j, double (&v)[VEC]) {
+      if constexpr (VEC == 2) {
+        if (have) {
+          const double2 x = __ldg(reinterpret_cast<const double2*>(a.T1 + j * ni + col));
+          v[0] = x.x; v[1] = x.y;
+        } else { v[0] = 0.0; v[1] = 0.0; }
+      } else {
+        v[0] = have ? ld_row(a.T1 + j * ni + col) : 0.0;
+      }
+    };
+    double up[VEC], cur[VEC], down[VEC];
+    load(j0 - 1, up);
+    load(j0, cur);
+    for (int64_t j = j0; j < j1; ++j) {
+      load(j + 1, down);
+      // left neighbour of my first column, right neighbour of my last column
+      double left = __shfl_up_sync(0xffffffffu, cur[VEC - 1], 1);
+      double right = __shfl_down_sync(0xffffffffu, cur[0], 1);
+      if (lane == 0 && col - 1 >= 0 && have) left = ld_row(a.T1 + j * ni + col - 1);
+      if (lane == 31 && col + VEC < ni) right = ld_row(a.T1 + j * ni + col + VEC);
+      double nv[VEC];
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) {
+        const double l = q == 0 ? left : cur[q - 1];
+        const double r = q == VEC - 1 ? right : cur[q + 1];
+        nv[q] = stencil(up[q], down[q], l, r);
+      }
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) {
+        const int64_t i = col + q;
+        if (i >= 1 && i < ni - 1) {
+          a.T2[j * ni + i] = nv[q];
+          err = O::combine(err, fabs(__dadd_rn(cur[q], -nv[q])));
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) { up[q] = cur[q]; cur[q] = down[q]; }
+    }
+  }
+  // a2 + a3: warp and CTA max, then a4: last CTA combines all CTA partials
+  err = block_reduce<OP_MAX, double, kBlock>(err, smem);
+  const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
+  if (threadIdx.x == 0) {
+    a.partials[cta] = err;
+    __threadfence();
+    const unsigned t = atomicAdd(a.tickets, 1u);
+    s_last = (t == (unsigned)(a.ntiles - 1));
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    double w = 0.0;
+    for (int64_t k = threadIdx.x; k < a.ntiles; k += kBlock) w = O::combine(w, ld_partial(a.partials + k));
+    w = block_reduce<OP_MAX, double, kBlock>(w, smem);
+    if (threadIdx.x == 0) {
+      *a.residual = w;
+      *a.tickets = 0u;
+    }
+  }
+}
+
+static int heat_launch(int64_t nj, int64_t ni, const double* T1, double* T2, double* residual,
+                       cudaStream_t s) {
+  const bool v2 = (ni % 2 == 0) && ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
+  const int strip = 32 * (v2 ? 2 : 1) * (kBlock / 32);
+  const int64_t gx = (ni + strip - 1) / strip;
+  const int64_t gy = nj > 2 ? (nj - 2 + kHeatRows - 1) / kHeatRows : 1;
+  if (gy > 65535) return XR_ERR_INVALID;
+  HeatArgs a;
+  a.T1 = T1; a.T2 = T2; a.residual = residual; a.nj = nj; a.ni = ni; a.ntiles = gx * gy;
+  void* partials = nullptr;
+  unsigned* tickets = nullptr;
+  int st = heat_workspace(s, a.ntiles * (int64_t)sizeof(double), 1, &partials, &tickets);
+  if (st) return st;
+  a.partials = static_cast<double*>(partials);
+  a.tickets = tickets;
+  dim3 grid((unsigned)gx, (unsigned)gy);
+  if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
+  else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);
+  count_launch();
+  if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  return XR_OK;
+}
+
+}  // namespace xr
+
+using namespace xr;
+
+extern "C" int xr_heat_step(int64_t nj, int64_t ni, const double* T1, double* T2, double* residual,
+                            xr_stream_t stream) {
+  if (nj < 0 || ni < 0) return XR_ERR_INVALID;
+  if (!residual) return XR_ERR_INVALID;
+  if ((nj * ni > 0) && (!T1 || !T2)) return XR_ERR_INVALID;
+  if (nj > 0 && ni > 0 && (nj > (INT64_MAX / 8) / ni)) return XR_ERR_INVALID;
+  if (T1 == T2 && nj * ni > 0) return XR_ERR_INVALID;
+  return heat_launch(nj, ni, T1, T2, residual, (cudaStream_t)stream);
+}
+
+extern "C" int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,
+                           double* residuals, xr_stream_t stream) {
+  if (iters < 0 || (iters > 0 && !residuals)) return XR_ERR_INVALID;
+  double* a = T1;
+  double* b = T2;
+  for (int64_t it = 0; it < iters; ++it) {
+    int st = xr_heat_step(nj, ni, a, b, residuals + it, stream);
+    if (st) return st;
+    double* t = a; a = b; b = t;
+  }
+  return XR_OK;
+}

@@ -1,0 +1,93 @@
+// xr_internal.h -- host <-> device interface shared by the library's own
+// translation units (never installed, never seen by the oracle).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace xr {
+
+constexpr int kBlock = 256;     // threads per CTA for every reduction kernel
+constexpr int kUnroll = 4;      // independent 16-B loads in flight per thread
+constexpr int kChainCap = 4096; // max sequential fp32 '+' chain per accumulator (C9)
+constexpr int kTargetCtasPerSm = 8;  // 2048 threads/SM at 256 threads/CTA
+
+enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4 };
+
+// Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]
+// -- covers R (O=1, C=1), KR (C=1) and RKR (C = outer reduced extent).
+struct SegArgs {
+  const void* in;
+  void* out;
+  void* partials;      // Acc[units] when splits > 1
+  unsigned* tickets;   // [O] when splits > 1, zero between launches
+  int64_t O, C, L, rowStride, oStride;
+  int64_t Sr, Sc;      // splits over rows and over columns; S = Sr*Sc per output
+  int64_t units;       // O * S
+  int init_from_out;
+};
+
+// Columns ("col"): out[b][c] = (+)_{r<R} in[b][r][c]  -- covers RK (B=1) and KRK.
+struct ColArgs {
+  const void* in;
+  void* out;
+  void* partials;      // Acc[B][tiles][S][32*vec] when S > 1
+  unsigned* tickets;   // [B][tiles]
+  int64_t B, R, K;
+  int64_t tiles, S;
+  int64_t units;       // B * tiles * S
+  int init_from_out;
+};
+
+// Elementwise: out[o] = init (+) in[o] (ident) or out[o] = init (fill).
+struct EltArgs {
+  const void* in;
+  void* out;
+  int64_t n;
+  int init_from_out;
+};
+
+struct Plan {
+  int shape = 0;        // xr_shape
+  int kernel = K_NONE;
+  int64_t cdims[3] = {0, 0, 0};
+  int64_t out_count = 0;
+  int group = 0;        // seg group width
+  int vec = 1;
+  int64_t splits = 1;
+  int64_t units = 0;
+  int block = kBlock;
+  int64_t ws_bytes = 0;
+  int64_t tickets = 0;
+  SegArgs seg{};
+  ColArgs col{};
+  EltArgs elt{};
+};
+
+// Pure host: validation happens before (api.cpp).  in_addr only matters for
+// its alignment (16-B vector path of the column kernel).
+void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
+               int num_sms, Plan* p);
+
+int dtype_size(int dtype);
+int acc_size(int op, int dtype);
+
+// Launch the plan's kernel (exactly one launch unless kernel == K_NONE); the
+// grid is min(units, num_sms * occupancy of the chosen kernel).
+cudaError_t launch_i32(int op, Plan& p, int num_sms, cudaStream_t s);
+cudaError_t launch_i64(int op, Plan& p, int num_sms, cudaStream_t s);
+cudaError_t launch_f32(int op, Plan& p, int num_sms, cudaStream_t s);
+cudaError_t launch_f64(int op, Plan& p, int num_sms, cudaStream_t s);
+
+// Fixed rank-order combine of nranks gathered partial results (each `n`
+// elements of dtype): out[i] = g[0][i] (+) g[1][i] (+) ... (sharded path).
+cudaError_t gather_i32(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+cudaError_t gather_i64(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+cudaError_t gather_f32(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+cudaError_t gather_f64(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+
+// Grid for `units` work items given the device's resident-CTA budget.
+int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm);
+
+void count_launch();
+
+}  // namespace xr

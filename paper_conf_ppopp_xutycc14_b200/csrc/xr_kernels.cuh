@@ -1,0 +1,405 @@
+// xr_kernels.cuh -- the reduction kernels (sm_100a), one family per canonical
+// shape (xr_plan.cpp).  Every launch is single pass: per-CTA (or per-warp)
+// partials are combined by the LAST unit to finish, found with an atomic
+// ticket after a __threadfence() -- the gang tier of SURVEY.md 8(a) a4, which
+// replaces the paper's "temporary buffer (partial in Figure 5(c)) ... then
+// another kernel ... is launched" (PAPER.md @24887-25280, 3.1.3) and the RMP
+// global buffer + second kernel (@29217-29414, @31388-31587).
+#pragma once
+#include <algorithm>
+
+#include "xr_internal.h"
+#include "xr_ops.cuh"
+
+namespace xr {
+
+// [lo, hi) of part `i` when n items are split in `parts` near-equal parts.
+__device__ __forceinline__ int64_t split_lo(int64_t n, int64_t parts, int64_t i) {
+  const int64_t q = n / parts, r = n % parts;
+  return i * q + (i < r ? i : r);
+}
+// Same, rounded down to a multiple of `v` (except the end, which is n).
+__device__ __forceinline__ int64_t split_lo_vec(int64_t n, int64_t parts, int64_t i, int v) {
+  if (i >= parts) return n;
+  return (split_lo(n, parts, i) / v) * v;
+}
+
+// ------------------------------------------------------------- a1 (rows)
+// Fold row[0..n) into the lane's private accumulators: a scalar head up to the
+// first 16-B boundary, 16-B vectors strided by the group width W with U loads
+// in flight, then a scalar tail.  Works for any dtype-aligned row start (the
+// paper's arbitrary iteration spaces, @33355-34930; reading C19).
+template <int OP, typename T, int W, int U>
+__device__ __forceinline__ void fold_row(const T* __restrict__ row, int64_t n, int lane,
+                                         typename Op<OP, T>::Acc (&acc)[U][16 / sizeof(T)]) {
+  using O = Op<OP, T>;
+  constexpr int VEC = 16 / sizeof(T);
+  int64_t head = (int64_t)((16u - ((uint32_t)(uintptr_t)row & 15u)) & 15u) / (int64_t)sizeof(T);
+  if (head > n) head = n;
+  if (lane < head) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(row + lane)));
+  row += head;
+  n -= head;
+  const int64_t nv = n / VEC;
+  const U128* __restrict__ vp = reinterpret_cast<const U128*>(row);
+  int64_t v = lane;
+  for (; v + (int64_t)(U - 1) * W < nv; v += (int64_t)U * W) {
+    U128 x[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) x[k] = ld_stream(vp + v + (int64_t)k * W);
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
+  }
+  for (; v < nv; v += W) {
+    const U128 x = ld_stream(vp + v);
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], O::lift(unpack<T>(x, q)));
+  }
+  const int64_t tail = n - nv * VEC;
+  if (lane < tail) acc[1 % U][0] = O::combine(acc[1 % U][0], O::lift(ld_scalar(row + nv * VEC + lane)));
+}
+
+// Combine the U x VEC private accumulators in a fixed pairwise order.
+template <int OP, typename T, int U, int VEC>
+__device__ __forceinline__ typename Op<OP, T>::Acc fold_acc(typename Op<OP, T>::Acc (&acc)[U][VEC]) {
+  using O = Op<OP, T>;
+#pragma unroll
+  for (int k = 1; k < U; ++k)
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], acc[k][q]);
+#pragma unroll
+  for (int w = VEC / 2; w > 0; w >>= 1)
+#pragma unroll
+    for (int q = 0; q < w; ++q) acc[0][q] = O::combine(acc[0][q], acc[0][q + w]);
+  return acc[0][0];
+}
+
+// This lane's partial over work unit u of a seg launch.
+template <int OP, typename T, int W, int U>
+__device__ __forceinline__ typename Op<OP, T>::Acc seg_unit(const SegArgs& a, int64_t u, int lane,
+                                                            int64_t* o_out) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  const int64_t S = a.Sr * a.Sc;
+  const int64_t o = u / S, s = u - o * S;
+  const int64_t sr = s / a.Sc, sc = s - sr * a.Sc;
+  const int64_t r0 = split_lo(a.C, a.Sr, sr), r1 = split_lo(a.C, a.Sr, sr + 1);
+  const int64_t c0 = split_lo_vec(a.L, a.Sc, sc, VEC), c1 = split_lo_vec(a.L, a.Sc, sc + 1, VEC);
+  Acc acc[U][VEC];
+#pragma unroll
+  for (int k = 0; k < U; ++k)
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[k][q] = O::identity();
+  const T* __restrict__ base = static_cast<const T*>(a.in) + o * a.oStride + c0;
+  for (int64_t r = r0; r < r1; ++r) fold_row<OP, T, W, U>(base + r * a.rowStride, c1 - c0, lane, acc);
+  *o_out = o;
+  return fold_acc<OP, T, U, VEC>(acc);
+}
+
+// a5: out[o] = init (+) R, init = identity or the prior out[o] (@21488-21990).
+template <int OP, typename T>
+__device__ __forceinline__ T merge_init(typename Op<OP, T>::Acc v, const T* out, int64_t o,
+                                        int init_from_out) {
+  using O = Op<OP, T>;
+  const typename O::Acc init = init_from_out ? O::lift(out[o]) : O::identity();
+  return O::finish(O::combine(init, v));
+}
+
+// ------------------------------------------------------------- seg kernel
+// Groups of W lanes (8 or 32: inside a warp; W == BLOCK: the whole CTA) each
+// reduce work units; a unit is (output o, split s).  Splits (S > 1) only
+// occur with W >= 32 (plan), so a ticket is always taken by a whole warp/CTA.
+template <int OP, typename T, int W, int BLOCK, int U>
+__global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  __shared__ Acc smem[32];
+  __shared__ int s_last;
+  T* out = static_cast<T*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  const int64_t S = a.Sr * a.Sc;
+
+  if constexpr (W == BLOCK) {
+    for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+      int64_t o;
+      Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
+      v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
+      if (S == 1) {
+        if (threadIdx.x == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+      } else {  // a4: gang tier, last CTA of output o combines its S partials
+        if (threadIdx.x == 0) {
+          partials[u] = v;
+          __threadfence();
+          const unsigned t = atomicAdd(&a.tickets[o], 1u);
+          s_last = (t == (unsigned)(S - 1));
+        }
+        __syncthreads();
+        if (s_last) {
+          __threadfence();
+          Acc w = O::identity();
+          for (int64_t i = threadIdx.x; i < S; i += BLOCK) w = O::combine(w, ld_partial(partials + o * S + i));
+          w = block_reduce<OP, T, BLOCK>(w, smem);
+          if (threadIdx.x == 0) {
+            out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+            a.tickets[o] = 0u;  // self-resetting for the next launch
+          }
+        }
+      }
+      __syncthreads();
+    }
+  } else {
+    static_assert(W <= 32 && (32 % W) == 0, "sub-warp group");
+    const int lane = threadIdx.x & (W - 1);
+    const int64_t gid = ((int64_t)blockIdx.x * BLOCK + threadIdx.x) / W;
+    const int64_t gid0 = gid - (int64_t)((threadIdx.x & 31) / W);  // first group of my warp
+    const int64_t G = (int64_t)gridDim.x * (BLOCK / W);
+    // warp-uniform trip count so every lane reaches the shuffles together
+    for (int64_t b = gid0; b < a.units; b += G) {
+      const int64_t u = b + (gid - gid0);
+      const bool active = u < a.units;
+      int64_t o = 0;
+      Acc v = active ? seg_unit<OP, T, W, U>(a, u, lane, &o) : O::identity();
+      v = group_reduce<OP, T, W>(v);
+      if (S == 1) {
+        if (active && lane == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+      } else {  // W == 32 here: the warp is one group, `active` is warp-uniform
+        int last = 0;
+        if (lane == 0) {
+          partials[u] = v;
+          __threadfence();
+          const unsigned t = atomicAdd(&a.tickets[o], 1u);
+          last = (t == (unsigned)(S - 1));
+        }
+        last = __shfl_sync(0xffffffffu, last, 0);
+        if (last) {
+          __threadfence();
+          Acc w = O::identity();
+          for (int64_t i = lane; i < S; i += 32) w = O::combine(w, ld_partial(partials + o * S + i));
+          w = group_reduce<OP, T, 32>(w);
+          if (lane == 0) {
+            out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+            a.tickets[o] = 0u;
+          }
+        }
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------- col kernel
+// Lanes own VEC contiguous kept columns (a 32*VEC-column tile per warp row);
+// the CTA's warps stride over the reduced rows of a row chunk; the worker tier
+// is a cross-warp combine of per-column partials in shared memory.
+template <int OP, typename T, int VEC, int BLOCK, int U>
+__global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int NW = BLOCK / 32;
+  constexpr int TW = 32 * VEC;
+  static_assert(TW <= BLOCK, "tile wider than the CTA");
+  __shared__ Acc sm[NW][TW];
+  __shared__ int s_last;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, t = threadIdx.x;
+  const T* __restrict__ in = static_cast<const T*>(a.in);
+  T* out = static_cast<T*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  const int64_t per_b = a.tiles * a.S;
+
+  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+    const int64_t b = u / per_b, rem = u - b * per_b;
+    const int64_t tile = rem / a.S, s = rem - tile * a.S;
+    const int64_t col = tile * TW + (int64_t)lane * VEC;
+    const int64_t r0 = split_lo(a.R, a.S, s), r1 = split_lo(a.R, a.S, s + 1);
+    Acc acc[U][VEC];
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[k][q] = O::identity();
+    if (col < a.K) {  // VEC path: K % VEC == 0, so the lane owns VEC whole columns
+      const T* __restrict__ base = in + b * a.R * a.K + col;
+      int64_t r = r0 + warp;
+      if constexpr (VEC > 1) {
+        for (; r + (int64_t)(U - 1) * NW < r1; r += (int64_t)U * NW) {
+          U128 x[U];
+#pragma unroll
+          for (int k = 0; k < U; ++k) x[k] = ld_stream(base + (r + (int64_t)k * NW) * a.K);
+#pragma unroll
+          for (int k = 0; k < U; ++k)
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
+        }
+        for (; r < r1; r += NW) {
+          const U128 x = ld_stream(base + r * a.K);
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], O::lift(unpack<T>(x, q)));
+        }
+      } else {
+        for (; r + (int64_t)(U - 1) * NW < r1; r += (int64_t)U * NW) {
+          T x[U];
+#pragma unroll
+          for (int k = 0; k < U; ++k) x[k] = ld_scalar(base + (r + (int64_t)k * NW) * a.K);
+#pragma unroll
+          for (int k = 0; k < U; ++k) acc[k][0] = O::combine(acc[k][0], O::lift(x[k]));
+        }
+        for (; r < r1; r += NW) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(base + r * a.K)));
+      }
+    }
+#pragma unroll
+    for (int k = 1; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], acc[k][q]);
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) sm[warp][lane * VEC + q] = acc[0][q];
+    __syncthreads();
+    // a3: worker tier, fixed warp order per column
+    Acc v = O::identity();
+    if (t < TW) {
+#pragma unroll
+      for (int w = 0; w < NW; ++w) v = O::combine(v, sm[w][t]);
+    }
+    const int64_t oc = tile * TW + t;
+    if (a.S == 1) {
+      if (t < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(v, out, b * a.K + oc, a.init_from_out);
+    } else {  // a4: gang tier per column tile
+      Acc* P = partials + (b * a.tiles + tile) * a.S * TW;
+      if (t < TW) P[s * TW + t] = v;
+      __threadfence();
+      __syncthreads();
+      if (t == 0) {
+        const unsigned tk = atomicAdd(&a.tickets[b * a.tiles + tile], 1u);
+        s_last = (tk == (unsigned)(a.S - 1));
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        Acc w2[VEC];
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) w2[q] = O::identity();
+        int64_t si = warp;
+        for (; si + 3 * NW < a.S; si += 4 * NW) {
+          Acc y[4][VEC];
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) y[k][q] = ld_partial(P + (si + k * NW) * TW + lane * VEC + q);
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) w2[q] = O::combine(w2[q], y[k][q]);
+        }
+        for (; si < a.S; si += NW)
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) w2[q] = O::combine(w2[q], ld_partial(P + si * TW + lane * VEC + q));
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) sm[warp][lane * VEC + q] = w2[q];
+        __syncthreads();
+        if (t < TW) {
+          Acc z = O::identity();
+#pragma unroll
+          for (int w = 0; w < NW; ++w) z = O::combine(z, sm[w][t]);
+          if (oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(z, out, b * a.K + oc, a.init_from_out);
+        }
+        if (t == 0) a.tickets[b * a.tiles + tile] = 0u;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ------------------------------------------------------------- elementwise
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
+  using O = Op<OP, T>;
+  const T* in = static_cast<const T*>(a.in);
+  T* out = static_cast<T*>(a.out);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = merge_init<OP, T>(O::lift(in[i]), out, i, a.init_from_out);
+}
+
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) fill_kernel(EltArgs a) {
+  using O = Op<OP, T>;
+  T* out = static_cast<T*>(a.out);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (int64_t)gridDim.x * blockDim.x)
+    out[i] = merge_init<OP, T>(O::identity(), out, i, a.init_from_out);
+}
+
+// Fixed rank-order combine of gathered partial results (sharded path).
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int nranks, int64_t n, T* out) {
+  using O = Op<OP, T>;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    typename O::Acc v = O::identity();
+    for (int r = 0; r < nranks; ++r) v = O::combine(v, O::lift(g[(int64_t)r * n + i]));
+    out[i] = O::finish(v);
+  }
+}
+
+// ------------------------------------------------------------- host launch
+template <typename K>
+static int occupancy(K kernel, int block) {
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kernel, block, 0) != cudaSuccess || n < 1) n = 1;
+  return n;
+}
+
+template <int OP, typename T>
+cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
+  constexpr int VEC = 16 / sizeof(T);
+  switch (p.kernel) {
+    case K_NONE:
+      return cudaSuccess;
+    case K_FILL: {
+      const int64_t grid = grid_for((p.elt.n + kBlock - 1) / kBlock, num_sms, 8);
+      fill_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(p.elt);
+      break;
+    }
+    case K_IDENT: {
+      const int64_t grid = grid_for((p.elt.n + kBlock - 1) / kBlock, num_sms, 8);
+      ident_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(p.elt);
+      break;
+    }
+    case K_SEG: {
+      const int64_t groups_per_cta = kBlock / p.group;
+      const int64_t ctas = (p.units + groups_per_cta - 1) / groups_per_cta;
+      if (p.group == 8) {
+        static int occ = occupancy(seg_kernel<OP, T, 8, kBlock, kUnroll>, kBlock);
+        seg_kernel<OP, T, 8, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+      } else if (p.group == 32) {
+        static int occ = occupancy(seg_kernel<OP, T, 32, kBlock, kUnroll>, kBlock);
+        seg_kernel<OP, T, 32, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+      } else {
+        static int occ = occupancy(seg_kernel<OP, T, kBlock, kBlock, kUnroll>, kBlock);
+        seg_kernel<OP, T, kBlock, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+      }
+      break;
+    }
+    case K_COL: {
+      if (p.vec == VEC && VEC > 1) {
+        static int occ = occupancy(col_kernel<OP, T, VEC, kBlock, kUnroll>, kBlock);
+        col_kernel<OP, T, VEC, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
+      } else {
+        static int occ = occupancy(col_kernel<OP, T, 1, kBlock, kUnroll>, kBlock);
+        col_kernel<OP, T, 1, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
+      }
+      break;
+    }
+    default:
+      return cudaErrorInvalidValue;
+  }
+  count_launch();
+  return cudaPeekAtLastError();
+}
+
+template <int OP, typename T>
+cudaError_t launch_gather_typed(const void* g, int nranks, int64_t n, void* out, cudaStream_t s) {
+  const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((n + kBlock - 1) / kBlock, 148 * 8));
+  gather_combine_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(static_cast<const T*>(g), nranks, n,
+                                                                  static_cast<T*>(out));
+  count_launch();
+  return cudaPeekAtLastError();
+}
+
+}  // namespace xr

@@ -1,0 +1,165 @@
+// xr_plan.cpp -- SURVEY.md 8(a) step a0: canonicalise (dims, level_mask) into
+// one of R / KR / RK / KRK / RKR / K and pick the kernel, group width, splits
+// and work units.  Pure host code (no CUDA calls), unit-tested on CPU through
+// xr_plan_describe.
+//
+// Why canonicalise: the paper binds levels to hardware (gang = blockIdx.x,
+// worker = threadIdx.y, vector = threadIdx.x; PAPER.md @11499-11699, 2.2), so
+// "memory coalescing is impossible in worker and gang partial reduction"
+// (@26577).  Here the API level is decoupled from the hardware tier: lanes
+// always run along the contiguous dimension, so every shape is coalesced.
+//  (1) drop every level of extent 1 (reducing or keeping one element is a
+//      no-op), (2) merge adjacent levels of the same status (row-major
+//      adjacent levels are one contiguous level), (3) the remaining pattern is
+//      one of R, KR, RK, KRK, RKR, K.
+#include <algorithm>
+
+#include "../../include/xreduce.h"
+#include "xr_internal.h"
+
+namespace xr {
+
+int dtype_size(int dtype) { return (dtype == XR_INT64 || dtype == XR_FP64) ? 8 : 4; }
+
+int acc_size(int op, int dtype) {
+  if (op == XR_OP_LAND || op == XR_OP_LOR) return 4;
+  return dtype_size(dtype);
+}
+
+static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
+  int64_t cap = (int64_t)std::max(num_sms, 1) * std::max(ctas_per_sm, 1);
+  return std::max<int64_t>(1, std::min(units, cap));
+}
+
+void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
+               int num_sms, Plan* p) {
+  *p = Plan();
+  const int size = dtype_size(dtype);
+  const int vec = 16 / size;
+  const int asz = acc_size(op, dtype);
+  const bool chain_capped = (op == XR_OP_ADD && dtype == XR_FP32);
+  const int64_t target_ctas = (int64_t)std::max(num_sms, 1) * kTargetCtasPerSm;
+
+  int64_t count = 1;
+  bool zero_reduced = false;
+  for (int d = 0; d < 3; ++d) {
+    const bool red = (mask >> d) & 1u;
+    if (!red) count *= dims[d];
+    else if (dims[d] == 0) zero_reduced = true;
+  }
+  p->out_count = count;
+  if (count == 0) {  // a kept extent of 0: empty output (C17)
+    p->shape = XR_SHAPE_NONE;
+    p->kernel = K_NONE;
+    return;
+  }
+  if (zero_reduced) {  // a reduced extent of 0: out = init (C17)
+    p->shape = XR_SHAPE_FILL;
+    p->kernel = K_FILL;
+    p->cdims[0] = count;
+    p->units = count;
+    p->elt.n = count;
+    return;
+  }
+
+  // (1) drop extent-1 levels, (2) merge adjacent levels of equal status
+  int64_t run_n[3];
+  bool run_red[3];
+  int nr = 0;
+  for (int d = 0; d < 3; ++d) {
+    if (dims[d] == 1) continue;
+    const bool red = (mask >> d) & 1u;
+    if (nr > 0 && run_red[nr - 1] == red) {
+      run_n[nr - 1] *= dims[d];
+    } else {
+      run_n[nr] = dims[d];
+      run_red[nr] = red;
+      ++nr;
+    }
+  }
+  for (int r = 0; r < nr; ++r) p->cdims[r] = run_n[r];
+
+  // (3) the pattern
+  if (nr == 0 || (nr == 1 && !run_red[0])) {  // K: every reduced extent is 1
+    p->shape = XR_SHAPE_IDENT;
+    p->kernel = K_IDENT;
+    p->cdims[0] = count;
+    p->units = count;
+    p->elt.n = count;
+    return;
+  }
+
+  const bool is_col = (nr == 2 && run_red[0]) || (nr == 3 && !run_red[0]);
+  if (is_col) {
+    // RK(R, K) or KRK(B, R, K): lanes own contiguous kept columns.
+    int64_t B = 1, R, K;
+    if (nr == 2) { R = run_n[0]; K = run_n[1]; p->shape = XR_SHAPE_RK; }
+    else { B = run_n[0]; R = run_n[1]; K = run_n[2]; p->shape = XR_SHAPE_KRK; }
+    const bool aligned = ((K * size) % 16 == 0) && (in_addr % 16 == 0);
+    const int cv = aligned ? vec : 1;
+    const int64_t TW = 32 * cv;
+    const int64_t tiles = cdiv(K, TW);
+    const int64_t NW = kBlock / 32;
+    int64_t S = 1;
+    const int64_t base = B * tiles;
+    if (base < 2 * target_ctas) {
+      S = cdiv(2 * target_ctas, base);
+      S = std::min<int64_t>(S, std::max<int64_t>(1, R / (NW * kUnroll)));
+      S = std::min<int64_t>(S, 1024);
+    }
+    if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * NW * kUnroll));
+    S = std::max<int64_t>(1, std::min<int64_t>(S, R));
+    p->kernel = K_COL;
+    p->vec = cv;
+    p->splits = S;
+    p->units = B * tiles * S;
+    p->group = kBlock;
+    if (S > 1) {
+      p->ws_bytes = B * tiles * S * TW * asz;
+      p->tickets = B * tiles;
+    }
+    ColArgs& c = p->col;
+    c.B = B; c.R = R; c.K = K; c.tiles = tiles; c.S = S; c.units = p->units;
+    return;
+  }
+
+  // seg: R(N) [O=1, C=1], KR(K, L) [C=1], RKR(R1, K, R2) [C=R1, rowStride=K*R2]
+  int64_t O, C, L, rowStride, oStride;
+  if (nr == 1) { O = 1; C = 1; L = run_n[0]; rowStride = 0; oStride = 0; p->shape = XR_SHAPE_R; }
+  else if (nr == 2) { O = run_n[0]; C = 1; L = run_n[1]; rowStride = 0; oStride = L; p->shape = XR_SHAPE_KR; }
+  else { O = run_n[1]; C = run_n[0]; L = run_n[2]; rowStride = O * L; oStride = L; p->shape = XR_SHAPE_RKR; }
+
+  const int64_t row_bytes = L * size;
+  int W = row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
+  auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
+  auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
+  const int64_t work = C * L;  // elements per output
+  int64_t S = 1;
+  if (O < 2 * resident_groups(W)) {
+    S = cdiv(2 * resident_groups(W), O);
+    S = std::min<int64_t>(S, std::max<int64_t>(1, work / min_unit_elems(W)));
+  }
+  if (chain_capped) S = std::max<int64_t>(S, cdiv(work, (int64_t)kChainCap * W * vec * kUnroll));
+  if (S > 1 && W < 32) W = 32;  // the gang-tier ticket runs per warp or per CTA
+  int64_t Sr, Sc;
+  if (C >= S) { Sr = S; Sc = 1; }
+  else { Sr = C; Sc = std::min<int64_t>(cdiv(S, C), std::max<int64_t>(1, L / vec)); }
+  S = Sr * Sc;
+
+  p->kernel = K_SEG;
+  p->group = W;
+  p->vec = vec;
+  p->splits = S;
+  p->units = O * S;
+  if (S > 1) {
+    p->ws_bytes = O * S * asz;
+    p->tickets = O;
+  }
+  SegArgs& s = p->seg;
+  s.O = O; s.C = C; s.L = L; s.rowStride = rowStride; s.oStride = oStride;
+  s.Sr = Sr; s.Sc = Sc; s.units = p->units;
+}
+
+}  // namespace xr

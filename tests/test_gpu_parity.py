@@ -1,0 +1,269 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, element by
+element, on seeded inputs shaped like the paper's workloads (DESIGN.md
+"Input recipe").  Sizes span several tiles and ragged tails; full BASELINE
+sizes are in test_gpu_fullsize.py."""
+import itertools
+import random
+
+import numpy as np
+import pytest
+
+import datagen
+from datagen import recipes
+import oracle
+from gpu_util import check, gpu_reduce
+
+pytestmark = pytest.mark.gpu
+
+ALL_MASKS = ["g", "w", "v", "gw", "gv", "wv", "gwv"]
+PAIRS = [(op, dt) for dt in ["int32", "int64", "fp32", "fp64"]
+         for op in ["+", "*", "max", "min", "&&", "||"] + (["&", "|", "^"] if dt.startswith("int") else [])]
+KIND = {"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "&": "band", "|": "bor",
+        "^": "bxor", "&&": "land", "||": "lor"}
+
+
+@pytest.fixture(scope="module", autouse=True)
+def lib():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    return xr
+
+
+# ---------------------------------------------------------------- config 1
+@pytest.mark.parametrize("levels", ["g", "w", "v", "gwv"])
+@pytest.mark.parametrize("variant", ["ints", "linear", "ones"])
+def test_cfg1_testsuite_nest(levels, variant):
+    dims = (64, 64, 128)
+    seed = datagen.case_seed(1, 0, 0, oracle.mask_of(levels), 1)
+    x = recipes.make(variant, dims, oracle.mask_of(levels), "int32", seed)
+    g = gpu_reduce("+", "int32", dims, levels, x)
+    check("+", "int32", dims, levels, g, x)
+    if variant == "linear" and levels == "gwv":
+        assert g.tolist() == [-262144]  # P1
+
+
+def test_cfg1_paper_literal_fig4():
+    """Fig 4 (a)/(b)/(c) with XR_INIT_FROM_OUT (P16)."""
+    NK, NJ, NI = 64, 64, 128
+    x = datagen.uniform_int(16, NK * NJ * NI, -1000, 1000, np.int32)
+    init_a = np.tile(np.arange(NJ, dtype=np.int32), NK)                       # i_sum = j
+    check("+", "int32", (NK, NJ, NI), "v", gpu_reduce("+", "int32", (NK, NJ, NI), "v", x, init_a), x, init_a)
+    init_b = np.repeat(np.arange(NK, dtype=np.int32), NI)                     # j_sum = k
+    check("+", "int32", (NK, NJ, NI), "w", gpu_reduce("+", "int32", (NK, NJ, NI), "w", x, init_b), x, init_b)
+    g = gpu_reduce("+", "int32", (NK, NJ, NI), "g", x)
+    assert g.reshape(NJ, NI)[0, 0] == int(x.reshape(NK, NJ, NI)[:, 0, 0].astype(np.int64).sum())
+
+
+# ---------------------------------------------------------------- op x dtype x mask
+@pytest.mark.parametrize("op,dtype", PAIRS)
+@pytest.mark.parametrize("dims", [(37, 41, 123), (3, 129, 1000), (130, 7, 33)])
+def test_all_pairs_all_masks(op, dtype, dims):
+    for levels in ALL_MASKS:
+        mask = oracle.mask_of(levels)
+        seed = datagen.case_seed(5, oracle.OPS[op], oracle.DTYPES[dtype], mask, sum(dims))
+        x = recipes.make(KIND[op], dims, mask, dtype, seed)
+        g = gpu_reduce(op, dtype, dims, levels, x)
+        check(op, dtype, dims, levels, g, x)
+
+
+@pytest.mark.parametrize("dtype", ["fp32", "fp64"])
+def test_fp_sums_exact_regime(dtype):
+    """Integer-valued data: any order is exact, so the GPU must be bit-exact (P8)."""
+    for dims in [(64, 64, 128), (5, 300, 701), (1000, 3, 17)]:
+        for levels in ALL_MASKS:
+            x = recipes.make("intvals", dims, 7, dtype, 88)
+            check("+", dtype, dims, levels, gpu_reduce("+", dtype, dims, levels, x), x, exact=True)
+
+
+@pytest.mark.parametrize("dtype", ["fp32", "fp64"])
+@pytest.mark.parametrize("kind", ["u01", "um11", "mulgen"])
+def test_fp_general_data(dtype, kind):
+    op = "*" if kind == "mulgen" else "+"
+    for dims in [(64, 64, 128), (17, 1000, 33)]:
+        for levels in ALL_MASKS:
+            x = recipes.make(kind, dims, 7, dtype, 123)
+            check(op, dtype, dims, levels, gpu_reduce(op, dtype, dims, levels, x), x)
+
+
+@pytest.mark.parametrize("dtype", ["fp32", "fp64"])
+def test_fp_products_exact_regime(dtype):
+    for dims in [(8, 64, 4096), (100, 300, 7)]:
+        for levels in ALL_MASKS:
+            x = recipes.make("mul", dims, oracle.mask_of(levels), dtype, 99)
+            check("*", dtype, dims, levels, gpu_reduce("*", dtype, dims, levels, x), x, exact=True)
+
+
+@pytest.mark.parametrize("dtype", ["fp32", "fp64"])
+@pytest.mark.parametrize("op", ["max", "min", "&&", "||", "+", "*"])
+def test_fp_special_values(op, dtype):
+    """NaN, +-inf, +-0 and subnormals (C7, C8): bit-exact for max/min/&&/||."""
+    for dims in [(33, 17, 65), (2, 2, 3000)]:
+        for levels in ALL_MASKS:
+            # products: specials on exact +-1/2/0.5 data; long U[-1,1) chains would
+            # underflow in dtype but not in the oracle's wider type (outside C10)
+            kind = "mulspecials" if op == "*" else "specials"
+            x = recipes.make(kind, dims, oracle.mask_of(levels), dtype, 7)
+            check(op, dtype, dims, levels, gpu_reduce(op, dtype, dims, levels, x), x)
+    z = np.array([-0.0, 0.0, -0.0], dtype=oracle.NP_DTYPES[dtype])
+    if op in ("max", "min"):
+        check(op, dtype, (3, 1, 1), "g", gpu_reduce(op, dtype, (3, 1, 1), "g", z), z)
+
+
+# ---------------------------------------------------------------- fuzz: ragged, misaligned
+def test_fuzz_shapes_and_misalignment():
+    rng = random.Random(2014)
+    sizes = [1, 2, 3, 31, 32, 33, 127, 128, 129, 1000, 4097]
+    for trial in range(120):
+        dims = tuple(rng.choice(sizes) for _ in range(3))
+        while np.prod(dims) > 3_000_000:
+            dims = tuple(rng.choice(sizes) for _ in range(3))
+        op, dtype = rng.choice(PAIRS)
+        levels = rng.choice(ALL_MASKS)
+        mask = oracle.mask_of(levels)
+        x = recipes.make(KIND[op], dims, mask, dtype, trial)
+        off = rng.randrange(0, 4)
+        init = None
+        if rng.random() < 0.4:
+            init = recipes.make(KIND[op], (oracle.out_count(dims, levels), 1, 1), 1, dtype, trial + 7)
+        g = gpu_reduce(op, dtype, dims, levels, x, init=init, offset=off)
+        check(op, dtype, dims, levels, g, x, init=init)
+
+
+@pytest.mark.parametrize("op,dtype", PAIRS)
+def test_init_from_out_every_pair(op, dtype):
+    dims = (9, 70, 130)
+    for levels in ALL_MASKS:
+        mask = oracle.mask_of(levels)
+        x = recipes.make(KIND[op], dims, mask, dtype, 5)
+        init = recipes.make("ints" if op not in ("&", "|", "^") else KIND[op],
+                            (oracle.out_count(dims, levels), 1, 1), 1, dtype, 6)
+        check(op, dtype, dims, levels, gpu_reduce(op, dtype, dims, levels, x, init=init), x, init=init)
+
+
+# ---------------------------------------------------------------- degenerate cases
+def test_empty_and_degenerate():
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    # reduced extent 0 -> out = init (C17); && normalises init to 0/1
+    init = np.arange(12, dtype=np.int32) - 3
+    for op in ["+", "*", "max", "min", "&&", "||", "^"]:
+        g = gpu_reduce(op, "int32", (4, 0, 3), "w", np.zeros(0, np.int32), init=init)
+        check(op, "int32", (4, 0, 3), "w", g, np.zeros(0, np.int32), init=init)
+        g2 = gpu_reduce(op, "int32", (4, 0, 3), "w", np.zeros(0, np.int32))
+        check(op, "int32", (4, 0, 3), "w", g2, np.zeros(0, np.int32))
+    # kept extent 0 -> nothing (status OK)
+    out = torch.zeros(1, dtype=torch.int32, device="cuda")
+    assert xr.xr_reduce("+", "int32", (0, 5, 5), "w", 0, out.data_ptr()) == 0
+    # all extents 1 / every reduced extent 1 (ident)
+    for dims, lv in [((1, 1, 1), "gwv"), ((5, 1, 7), "w"), ((1, 9, 11), "g")]:
+        x = datagen.uniform_int(3, int(np.prod(dims)), -9, 9, np.int32)
+        init = datagen.uniform_int(4, oracle.out_count(dims, lv), -9, 9, np.int32)
+        check("+", "int32", dims, lv, gpu_reduce("+", "int32", dims, lv, x, init=init), x, init=init)
+        check("&&", "int32", dims, lv, gpu_reduce("&&", "int32", dims, lv, x), x)
+    # unsupported + invalid map to exceptions in the binding
+    with pytest.raises(xr.XReduceError) as e:
+        xr.reduce(torch.ones(8, device="cuda"), "&", "gwv")
+    assert e.value.status == xr.ERR_UNSUPPORTED
+
+
+def test_binding_reduce_shapes():
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    t = torch.arange(2 * 3 * 4, dtype=torch.int64, device="cuda").reshape(2, 3, 4)
+    assert xr.reduce(t, "+", "v").shape == (2, 3)
+    assert xr.reduce(t, "+", "gw").cpu().tolist() == t.sum((0, 1)).cpu().tolist()
+    assert xr.reduce(t, "max", "gwv").item() == 23
+    assert xr.reduce(t, "+", "v", init=torch.ones(2, 3, dtype=torch.int64)).cpu().tolist() == \
+        (t.sum(2) + 1).cpu().tolist()
+
+
+def test_deterministic_and_streams():
+    """Fixed grids -> bit-identical fp results run to run; two streams at once."""
+    import torch
+    x = recipes.make("u01", (1, 1, 1 << 24), 4, "fp32", 1)
+    a = gpu_reduce("+", "fp32", (1, 1, 1 << 24), "gwv", x)
+    b = gpu_reduce("+", "fp32", (1, 1, 1 << 24), "gwv", x)
+    assert a.view(np.uint32)[0] == b.view(np.uint32)[0]
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    y = recipes.make("um11", (64, 512, 512), 7, "fp32", 2)
+    r1 = gpu_reduce("+", "fp32", (64, 512, 512), "gw", y, stream=s1)
+    r2 = gpu_reduce("max", "fp32", (64, 512, 512), "v", y, stream=s2)
+    check("+", "fp32", (64, 512, 512), "gw", r1, y)
+    check("max", "fp32", (64, 512, 512), "v", r2, y)
+
+
+def test_host_buffer_path():
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    for op, dtype, dims, lv in [("+", "fp64", (300, 40, 77), "wv"), ("^", "int64", (5, 6, 100001), "v"),
+                                ("min", "fp32", (1 << 20, 1, 1), "gwv")]:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, 3)
+        out = np.zeros(oracle.out_count(dims, lv), oracle.NP_DTYPES[dtype])
+        assert xr.xr_reduce_host(op, dtype, dims, lv, x.ctypes.data, out.ctypes.data) == 0
+        check(op, dtype, dims, lv, out, x)
+
+
+def test_launch_count_single_pass():
+    """Exactly one kernel launch per xr_reduce call (no second launch)."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    x = torch.rand(1 << 22, device="cuda")
+    xr.reduce(x, "+", "gwv")
+    torch.cuda.synchronize()
+    n0 = xr.xr_launch_count()
+    for lv in ["g", "w", "v", "gw", "gv", "wv", "gwv"]:
+        xr.reduce(x, "+", lv, nest=(64, 256, 256))
+    torch.cuda.synchronize()
+    assert xr.xr_launch_count() - n0 == 7
+
+
+# ---------------------------------------------------------------- heat (config 4)
+@pytest.mark.parametrize("nj,ni", [(8, 8), (130, 258), (67, 131), (3, 40), (300, 64)])
+def test_heat_bitwise(nj, ni):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    iters = 25
+    T0 = oracle.heat_init(nj, ni)
+    ref_T, ref_res = oracle.heat(nj, ni, iters, T0)
+    t1 = torch.from_numpy(T0).cuda()
+    t2 = t1.clone()
+    res = torch.zeros(iters, dtype=torch.float64, device="cuda")
+    assert xr.xr_heat_run(nj, ni, iters, t1.data_ptr(), t2.data_ptr(), res.data_ptr(),
+                          torch.cuda.current_stream().cuda_stream) == 0
+    torch.cuda.synchronize()
+    final = (t1 if iters % 2 == 0 else t2).cpu().numpy()
+    assert res.cpu().numpy().tolist() == ref_res.tolist()
+    assert np.array_equal(final.view(np.uint64), ref_T.view(np.uint64))
+    if nj >= 6 and ni >= 6:
+        assert res.cpu().numpy()[:3].tolist() == [0.25, 0.125, 0.078125]
+
+
+# ---------------------------------------------------------------- sharded (single-device sim)
+@pytest.mark.parametrize("op,dtype", [("+", "int64"), ("^", "int32"), ("max", "fp32"), ("&&", "fp64"),
+                                      ("*", "int32"), ("+", "fp32"), ("|", "int64")])
+def test_sharded_sim_matches_unsharded(op, dtype):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    G = 4
+    local = (16, 12, 100)
+    gdims = (local[0] * G, local[1], local[2])
+    for levels in ALL_MASKS:
+        mask = oracle.mask_of(levels)
+        x = recipes.make(KIND[op], gdims, mask, dtype, 42)
+        xs = torch.from_numpy(x).cuda()
+        n_loc = int(np.prod(local))
+        shards = [xs[r * n_loc:(r + 1) * n_loc] for r in range(G)]
+        info = xr.xr_shard_plan(op, dtype, local, mask, G, 0)
+        for with_init in (False, True):
+            m = mask
+            init = None
+            out = torch.zeros(info["global_count"], dtype=xs.dtype, device="cuda")
+            if with_init:
+                init = recipes.make("ints", (info["global_count"], 1, 1), 1, dtype, 9)
+                out.copy_(torch.from_numpy(init))
+                m |= xr.INIT_FROM_OUT
+            st = xr.xr_reduce_sharded_sim(op, dtype, local, m, [s.data_ptr() for s in shards],
+                                          out.data_ptr(), torch.cuda.current_stream().cuda_stream)
+            assert st == 0
+            torch.cuda.synchronize()
+            check(op, dtype, gdims, levels, out.cpu().numpy(), x, init=init)
