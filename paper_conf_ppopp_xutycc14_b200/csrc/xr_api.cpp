@@ -139,8 +139,13 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   make_plan(op, dtype, dims, mask & 7u, (uint64_t)(uintptr_t)in, sms, &p);
   if (p.kernel == K_NONE) return XR_OK;
   Workspace& w = g_ws[{dev, (uintptr_t)stream}];
-  st = ensure_ws(w, p.ws_bytes, p.tickets, stream);
+  // tickets are followed by the two 64-bit scheduler counters (8-B aligned)
+  const int64_t tick_words = (p.tickets + 1) & ~int64_t(1);
+  st = ensure_ws(w, p.ws_bytes, tick_words + (p.sched ? 4 : 0), stream);
   if (st) return st;
+  unsigned long long* sched = reinterpret_cast<unsigned long long*>(w.tickets + tick_words);
+  p.seg.sched = sched;
+  p.col.sched = sched;
   const int ifo = (mask & XR_INIT_FROM_OUT) ? 1 : 0;
   p.seg.in = in; p.seg.out = out; p.seg.partials = w.partials; p.seg.tickets = w.tickets;
   p.seg.init_from_out = ifo;
@@ -226,6 +231,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   info->units = p.units;
   info->block = p.block;
   int64_t ctas = p.units;
+  if (p.kernel == K_STREAM) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);
@@ -247,7 +253,8 @@ int xr_reserve(int op, int dtype, const int64_t nest_dims[3], unsigned level_mas
   Plan q;
   make_plan(op, dtype, nest_dims, level_mask & 7u, 4, device_sms(dev), &q);
   Workspace& w = g_ws[{dev, (uintptr_t)stream}];
-  return ensure_ws(w, std::max(p.ws_bytes, q.ws_bytes), std::max(p.tickets, q.tickets), (cudaStream_t)stream);
+  const int64_t words = std::max((p.tickets + 1) & ~int64_t(1), (q.tickets + 1) & ~int64_t(1)) + 4;
+  return ensure_ws(w, std::max(p.ws_bytes, q.ws_bytes), words, (cudaStream_t)stream);
 }
 
 int xr_shutdown(void) {

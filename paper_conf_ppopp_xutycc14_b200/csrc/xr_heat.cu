@@ -21,7 +21,8 @@ namespace xr {
 
 int heat_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets);
 
-constexpr int kHeatRows = 32;  // rows marched per warp
+constexpr int kHeatRows = 64;     // rows marched per warp (halo re-read: 2/64)
+constexpr int kHeatPrefetch = 4;  // rows in flight per lane
 
 struct HeatArgs {
   const double* T1;
@@ -40,11 +41,17 @@ __device__ __forceinline__ double stencil(double up, double down, double left, d
 __device__ __forceinline__ double ld_row(const double* p) { return __ldg(p); }
 
 // VEC = columns per lane (2: 16-B loads, needs ni even and 16-B aligned rows).
+// Each warp marches down kHeatRows rows of a 32*VEC-column strip.  Rows are
+// loaded PF rows ahead into a register ring (static indices via full unroll),
+// so every lane keeps PF independent 16-B loads in flight: the sweep is an
+// HBM stream, and one load per lane per row left it latency bound (68% of
+// peak in profiles/ r01).
 template <int VEC>
 __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
   using O = Op<OP_MAX, double>;
   constexpr int NW = kBlock / 32;
   constexpr int STRIP = 32 * VEC;
+  constexpr int PF = kHeatPrefetch;
   __shared__ double smem[32];
   __shared__ int s_last;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -57,43 +64,62 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
 
   if (j0 < j1 && c0 < ni) {
     const bool have = col < ni;
+    const double* base = a.T1 + col;
+    // rows past j1 (the last one this warp needs) are never read
     auto load = [&](int64_t j, double (&v)[VEC]) {
-      if constexpr (VEC == 2) {
-        if (have) {
-          const double2 x = __ldg(reinterpret_cast<const double2*>(a.T1 + j * ni + col));
-          v[0] = x.x; v[1] = x.y;
-        } else { v[0] = 0.0; v[1] = 0.0; }
+      if (have && j <= j1) {
+        if constexpr (VEC == 2) {
+          const double2 x = __ldg(reinterpret_cast<const double2*>(base + j * ni));
+          v[0] = x.x;
+          v[1] = x.y;
+        } else {
+          v[0] = ld_row(base + j * ni);
+        }
       } else {
-        v[0] = have ? ld_row(a.T1 + j * ni + col) : 0.0;
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) v[q] = 0.0;
       }
     };
-    double up[VEC], cur[VEC], down[VEC];
+    double up[VEC], cur[VEC], ring[PF][VEC];
     load(j0 - 1, up);
     load(j0, cur);
-    for (int64_t j = j0; j < j1; ++j) {
-      load(j + 1, down);
-      // left neighbour of my first column, right neighbour of my last column
-      double left = __shfl_up_sync(0xffffffffu, cur[VEC - 1], 1);
-      double right = __shfl_down_sync(0xffffffffu, cur[0], 1);
-      if (lane == 0 && col - 1 >= 0 && have) left = ld_row(a.T1 + j * ni + col - 1);
-      if (lane == 31 && col + VEC < ni) right = ld_row(a.T1 + j * ni + col + VEC);
-      double nv[VEC];
 #pragma unroll
-      for (int q = 0; q < VEC; ++q) {
-        const double l = q == 0 ? left : cur[q - 1];
-        const double r = q == VEC - 1 ? right : cur[q + 1];
-        nv[q] = stencil(up[q], down[q], l, r);
-      }
+    for (int k = 0; k < PF; ++k) load(j0 + 1 + k, ring[k]);
+    for (int64_t jb = j0; jb < j1; jb += PF) {
+      double next[PF][VEC];
 #pragma unroll
-      for (int q = 0; q < VEC; ++q) {
-        const int64_t i = col + q;
-        if (i >= 1 && i < ni - 1) {
-          a.T2[j * ni + i] = nv[q];
-          err = O::combine(err, fabs(__dadd_rn(cur[q], -nv[q])));
+      for (int k = 0; k < PF; ++k) load(jb + 1 + PF + k, next[k]);  // next group in flight
+#pragma unroll
+      for (int k = 0; k < PF; ++k) {
+        const int64_t j = jb + k;
+        if (j < j1) {  // warp-uniform
+          // left neighbour of my first column, right neighbour of my last column
+          double left = __shfl_up_sync(0xffffffffu, cur[VEC - 1], 1);
+          double right = __shfl_down_sync(0xffffffffu, cur[0], 1);
+          if (lane == 0 && col >= 1 && have) left = ld_row(base + j * ni - 1);
+          if (lane == 31 && col + VEC < ni) right = ld_row(base + j * ni + VEC);
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) {
+            const double l = q == 0 ? left : cur[q - 1];
+            const double r = q == VEC - 1 ? right : cur[q + 1];
+            const double nv = stencil(up[q], ring[k][q], l, r);
+            const int64_t i = col + q;
+            if (i >= 1 && i < ni - 1) {
+              __stcs(a.T2 + j * ni + i, nv);
+              err = O::combine(err, fabs(__dadd_rn(cur[q], -nv)));
+            }
+          }
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) {
+            up[q] = cur[q];
+            cur[q] = ring[k][q];
+          }
         }
       }
 #pragma unroll
-      for (int q = 0; q < VEC; ++q) { up[q] = cur[q]; cur[q] = down[q]; }
+      for (int k = 0; k < PF; ++k)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) ring[k][q] = next[k][q];
     }
   }
   // a2 + a3: warp and CTA max, then a4: last CTA combines all CTA partials

@@ -10,8 +10,12 @@ constexpr int kBlock = 256;     // threads per CTA for every reduction kernel
 constexpr int kUnroll = 4;      // independent 16-B loads in flight per thread
 constexpr int kChainCap = 4096; // max sequential fp32 '+' chain per accumulator (C9)
 constexpr int kTargetCtasPerSm = 8;  // 2048 threads/SM at 256 threads/CTA
+constexpr int kUnitsPerCta = 8;      // dynamic units per resident CTA (tail balance)
 
-enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4 };
+enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5 };
+
+constexpr int kStages = 4;          // bulk-copy ring depth (stream kernel)
+constexpr int kStageBytes = 16384;  // bytes per stage
 
 // Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]
 // -- covers R (O=1, C=1), KR (C=1) and RKR (C = outer reduced extent).
@@ -20,6 +24,7 @@ struct SegArgs {
   void* out;
   void* partials;      // Acc[units] when splits > 1
   unsigned* tickets;   // [O] when splits > 1, zero between launches
+  unsigned long long* sched;  // [2] dynamic unit counter + exit counter (CTA-wide groups)
   int64_t O, C, L, rowStride, oStride;
   int64_t Sr, Sc;      // splits over rows and over columns; S = Sr*Sc per output
   int64_t units;       // O * S
@@ -32,6 +37,7 @@ struct ColArgs {
   void* out;
   void* partials;      // Acc[B][tiles][S][32*vec] when S > 1
   unsigned* tickets;   // [B][tiles]
+  unsigned long long* sched;  // [2] dynamic unit counter + exit counter
   int64_t B, R, K;
   int64_t tiles, S;
   int64_t units;       // B * tiles * S
@@ -58,6 +64,7 @@ struct Plan {
   int block = kBlock;
   int64_t ws_bytes = 0;
   int64_t tickets = 0;
+  bool sched = false;   // CTA-wide units are claimed dynamically (2 extra counters)
   SegArgs seg{};
   ColArgs col{};
   EltArgs elt{};

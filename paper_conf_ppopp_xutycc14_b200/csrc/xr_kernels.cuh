@@ -107,6 +107,40 @@ __device__ __forceinline__ T merge_init(typename Op<OP, T>::Acc v, const T* out,
   return O::finish(O::combine(init, v));
 }
 
+// Fold p[start], p[start+stride], ... (< n) with 8 independent L2 loads in
+// flight per round (the last-CTA combine is latency bound, not bandwidth bound).
+template <int OP, typename T>
+__device__ __forceinline__ typename Op<OP, T>::Acc fold_partials(const typename Op<OP, T>::Acc* p, int64_t n,
+                                                                 int64_t start, int64_t stride) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  Acc w = O::identity();
+  int64_t i = start;
+  for (; i + 7 * stride < n; i += 8 * stride) {
+    Acc y[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) y[k] = ld_partial(p + i + k * stride);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) w = O::combine(w, y[k]);
+  }
+  for (; i < n; i += stride) w = O::combine(w, ld_partial(p + i));
+  return w;
+}
+
+// Dynamic unit claiming for CTA-wide work: thread 0 fetches the next unit
+// index (prefetched one unit ahead into a parity slot) from a device counter;
+// the last CTA to exit resets the counters for the next launch.
+__device__ __forceinline__ void sched_exit(unsigned long long* c) {
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long t = atomicAdd(c + 1, 1ull);
+    if (t == (unsigned long long)gridDim.x - 1ull) {
+      c[0] = 0ull;
+      c[1] = 0ull;
+    }
+  }
+}
+
 // ------------------------------------------------------------- seg kernel
 // Groups of W lanes (8 or 32: inside a warp; W == BLOCK: the whole CTA) each
 // reduce work units; a unit is (output o, split s).  Splits (S > 1) only
@@ -122,7 +156,13 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
   const int64_t S = a.Sr * a.Sc;
 
   if constexpr (W == BLOCK) {
-    for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+    __shared__ long long s_unit[2];
+    if (threadIdx.x == 0) s_unit[0] = (long long)atomicAdd(a.sched, 1ull);
+    __syncthreads();
+    long long u = s_unit[0];
+    int par = 1;
+    while (u < a.units) {
+      if (threadIdx.x == 0) s_unit[par] = (long long)atomicAdd(a.sched, 1ull);  // next, in flight
       int64_t o;
       Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
       v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
@@ -138,8 +178,7 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
         __syncthreads();
         if (s_last) {
           __threadfence();
-          Acc w = O::identity();
-          for (int64_t i = threadIdx.x; i < S; i += BLOCK) w = O::combine(w, ld_partial(partials + o * S + i));
+          Acc w = fold_partials<OP, T>(partials + o * S, S, threadIdx.x, BLOCK);
           w = block_reduce<OP, T, BLOCK>(w, smem);
           if (threadIdx.x == 0) {
             out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
@@ -148,7 +187,10 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
         }
       }
       __syncthreads();
+      u = s_unit[par];
+      par ^= 1;
     }
+    sched_exit(a.sched);
   } else {
     static_assert(W <= 32 && (32 % W) == 0, "sub-warp group");
     const int lane = threadIdx.x & (W - 1);
@@ -175,8 +217,7 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
         last = __shfl_sync(0xffffffffu, last, 0);
         if (last) {
           __threadfence();
-          Acc w = O::identity();
-          for (int64_t i = lane; i < S; i += 32) w = O::combine(w, ld_partial(partials + o * S + i));
+          Acc w = fold_partials<OP, T>(partials + o * S, S, lane, 32);
           w = group_reduce<OP, T, 32>(w);
           if (lane == 0) {
             out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
@@ -186,6 +227,164 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
       }
     }
   }
+}
+
+// ------------------------------------------------------------- stream kernel
+// R and long-row KR shapes (C == 1): each unit is one contiguous range.  Its
+// 16-B-aligned body is streamed into a ring of NS shared-memory stages by the
+// TMA bulk-copy engine (cp.async.bulk, completion on an mbarrier with a byte
+// count); thread 0 is the producer and keeps NS stages (NS*STAGE bytes) in
+// flight ACROSS unit boundaries, so memory-level parallelism no longer depends
+// on registers or per-element ALU cost.  All threads fold the stage from
+// shared memory (a1), then the warp / CTA / last-CTA tiers run as in seg.
+struct StreamGeom {
+  int64_t o;
+  int64_t head, nbody, tail;  // elements
+  const void* row;
+};
+
+template <typename T>
+__device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u) {
+  constexpr int VEC = 16 / sizeof(T);
+  StreamGeom g;
+  const int64_t S = a.Sc;
+  g.o = u / S;
+  const int64_t s = u - g.o * S;
+  const int64_t c0 = split_lo_vec(a.L, S, s, VEC), c1 = split_lo_vec(a.L, S, s + 1, VEC);
+  const T* row = static_cast<const T*>(a.in) + g.o * a.oStride + c0;
+  const int64_t n = c1 - c0;
+  int64_t head = (int64_t)((16u - ((uint32_t)(uintptr_t)row & 15u)) & 15u) / (int64_t)sizeof(T);
+  if (head > n) head = n;
+  g.head = head;
+  g.nbody = ((n - head) / VEC) * VEC;
+  g.tail = n - head - g.nbody;
+  g.row = row;
+  return g;
+}
+
+template <int OP, typename T, int BLOCK, int NS, int STAGE>
+__global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int PER = STAGE / (16 * BLOCK);  // 16-B vectors per thread per stage
+  constexpr int RING = 8;                    // published unit ids (producer <= 3 units ahead)
+  static_assert(PER >= 1 && STAGE % (16 * BLOCK) == 0, "stage geometry");
+  extern __shared__ __align__(128) unsigned char stage_mem[];  // NS * STAGE
+  __shared__ __align__(8) uint64_t full[NS];
+  __shared__ long long s_units[RING];
+  __shared__ Acc smem[32];
+  __shared__ int s_last;
+  const int tid = threadIdx.x;
+  T* out = static_cast<T*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  const int64_t S = a.Sc;
+
+  // ---- producer state (meaningful in thread 0 only)
+  long long p_unit = 0, p_next = 0;
+  int64_t p_k = 0, p_nk = 0, p_bytes = 0, g_issue = 0;
+  const char* p_src = nullptr;
+  int p_seq = 0;
+  auto p_start = [&](long long u) {
+    p_unit = u;
+    s_units[p_seq & (RING - 1)] = u < a.units ? u : -1;
+    ++p_seq;
+    p_k = 0;
+    p_nk = 0;
+    if (u < a.units) {
+      const StreamGeom g = stream_geom<T>(a, u);
+      p_src = static_cast<const char*>(g.row) + g.head * (int64_t)sizeof(T);
+      p_bytes = g.nbody * (int64_t)sizeof(T);
+      p_nk = (p_bytes + STAGE - 1) / STAGE;
+    }
+  };
+  auto p_issue = [&]() {  // issue the next chunk of the global chunk sequence, if any
+    while (p_unit < a.units && p_k == p_nk) {
+      const long long nu = p_next;
+      p_next = (long long)atomicAdd(a.sched, 1ull);  // claimed one unit ahead
+      p_start(nu);
+    }
+    if (p_unit >= a.units) return;
+    const int slot = (int)(g_issue % NS);
+    const unsigned bytes = (unsigned)min((int64_t)STAGE, p_bytes - p_k * STAGE);
+    mbar_expect_tx(&full[slot], bytes);
+    bulk_g2s(stage_mem + slot * STAGE, p_src + p_k * STAGE, bytes, &full[slot]);
+    ++p_k;
+    ++g_issue;
+  };
+
+  if (tid == 0) {
+#pragma unroll
+    for (int k = 0; k < NS; ++k) mbar_init(&full[k], 1);
+    fence_mbar_init();
+    const long long u0 = (long long)atomicAdd(a.sched, 1ull);
+    p_next = (long long)atomicAdd(a.sched, 1ull);
+    p_start(u0);
+    for (int k = 0; k < NS; ++k) p_issue();
+  }
+  __syncthreads();
+
+  int seq = 0;
+  int64_t g = 0;  // consumer's global chunk index (stage = g % NS, phase parity = (g / NS) & 1)
+  while (true) {
+    const long long u = s_units[seq & (RING - 1)];
+    if (u < 0) break;
+    const StreamGeom geo = stream_geom<T>(a, u);
+    const T* row = static_cast<const T*>(geo.row);
+    Acc acc[PER][VEC];
+#pragma unroll
+    for (int j = 0; j < PER; ++j)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
+    if (tid < geo.head) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(row + tid)));
+    if (tid < geo.tail)
+      acc[0][VEC - 1] = O::combine(acc[0][VEC - 1], O::lift(ld_scalar(row + geo.head + geo.nbody + tid)));
+    const int64_t body_bytes = geo.nbody * (int64_t)sizeof(T);
+    const int64_t nk = (body_bytes + STAGE - 1) / STAGE;
+    for (int64_t k = 0; k < nk; ++k, ++g) {
+      const int slot = (int)(g % NS);
+      mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      const int64_t bytes = min((int64_t)STAGE, body_bytes - k * STAGE);
+      const unsigned char* st = stage_mem + slot * STAGE;
+#pragma unroll
+      for (int j = 0; j < PER; ++j) {
+        const int off = (tid + j * BLOCK) * 16;
+        if (off < bytes) {
+          const U128 x = *reinterpret_cast<const U128*>(st + off);
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x, q)));
+        }
+      }
+      __syncthreads();            // every thread is done with this stage
+      if (tid == 0) p_issue();    // refill it NS chunks ahead
+    }
+    Acc v = fold_acc<OP, T, PER, VEC>(acc);
+    v = block_reduce<OP, T, BLOCK>(v, smem);
+    const int64_t o = geo.o;
+    if (S == 1) {
+      if (tid == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+    } else {
+      if (tid == 0) {
+        partials[u] = v;
+        __threadfence();
+        const unsigned t = atomicAdd(&a.tickets[o], 1u);
+        s_last = (t == (unsigned)(S - 1));
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        Acc w = fold_partials<OP, T>(partials + o * S, S, tid, BLOCK);
+        w = block_reduce<OP, T, BLOCK>(w, smem);
+        if (tid == 0) {
+          out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+          a.tickets[o] = 0u;
+        }
+      }
+    }
+    __syncthreads();
+    ++seq;
+  }
+  sched_exit(a.sched);
 }
 
 // ------------------------------------------------------------- col kernel
@@ -207,7 +406,13 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
   Acc* partials = static_cast<Acc*>(a.partials);
   const int64_t per_b = a.tiles * a.S;
 
-  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+  __shared__ long long s_unit[2];
+  if (t == 0) s_unit[0] = (long long)atomicAdd(a.sched, 1ull);
+  __syncthreads();
+  long long u = s_unit[0];
+  int par = 1;
+  while (u < a.units) {
+    if (t == 0) s_unit[par] = (long long)atomicAdd(a.sched, 1ull);  // next unit, in flight
     const int64_t b = u / per_b, rem = u - b * per_b;
     const int64_t tile = rem / a.S, s = rem - tile * a.S;
     const int64_t col = tile * TW + (int64_t)lane * VEC;
@@ -305,7 +510,10 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
       }
     }
     __syncthreads();
+    u = s_unit[par];
+    par ^= 1;
   }
+  sched_exit(a.sched);
 }
 
 // ------------------------------------------------------------- elementwise
@@ -374,6 +582,18 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
         static int occ = occupancy(seg_kernel<OP, T, kBlock, kBlock, kUnroll>, kBlock);
         seg_kernel<OP, T, kBlock, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
       }
+      break;
+    }
+    case K_STREAM: {
+      auto kern = stream_kernel<OP, T, kBlock, kStages, kStageBytes>;
+      constexpr int dyn = kStages * kStageBytes;
+      static int occ = [&] {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        return n;
+      }();
+      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_COL: {

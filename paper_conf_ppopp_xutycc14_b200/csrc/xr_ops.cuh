@@ -44,10 +44,6 @@ template <> __device__ __forceinline__ int64_t highest<int64_t>() { return INT64
 template <> __device__ __forceinline__ float highest<float>() { return __int_as_float(0x7f800000u); }
 template <> __device__ __forceinline__ double highest<double>() { return __longlong_as_double(0x7ff0000000000000ull); }
 
-__device__ __forceinline__ bool sign_bit(float x) { return __float_as_uint(x) >> 31; }
-__device__ __forceinline__ bool sign_bit(double x) {
-  return static_cast<unsigned long long>(__double_as_longlong(x)) >> 63;
-}
 
 // Op traits.  Acc is the accumulator type:
 //   int  + * & | ^ : unsigned of the same width (two's-complement wrap, C6)
@@ -111,23 +107,33 @@ template <typename T> struct Op<OP_MUL, T, true> {
 };
 // ---- floating point: max min, reading C7 (C fmax/fmin: a NaN operand is
 // ignored; -0 < +0 so the result is order independent and bit exact).
+// Branch-free: FMNMX already ignores a NaN operand; numerically equal operands
+// (only a +-0 pair can differ in bits) combine by AND (max: +0 wins) or OR
+// (min: -0 wins) of their bit patterns.
+__device__ __forceinline__ float bits_and(float a, float b) { return __uint_as_float(__float_as_uint(a) & __float_as_uint(b)); }
+__device__ __forceinline__ float bits_or(float a, float b) { return __uint_as_float(__float_as_uint(a) | __float_as_uint(b)); }
+__device__ __forceinline__ double bits_and(double a, double b) {
+  return __longlong_as_double(__double_as_longlong(a) & __double_as_longlong(b));
+}
+__device__ __forceinline__ double bits_or(double a, double b) {
+  return __longlong_as_double(__double_as_longlong(a) | __double_as_longlong(b));
+}
+__device__ __forceinline__ float hw_max(float a, float b) { return fmaxf(a, b); }
+__device__ __forceinline__ double hw_max(double a, double b) { return fmax(a, b); }
+__device__ __forceinline__ float hw_min(float a, float b) { return fminf(a, b); }
+__device__ __forceinline__ double hw_min(double a, double b) { return fmin(a, b); }
 template <typename T> struct Op<OP_MAX, T, true> {
   using Acc = T;
   static __device__ __forceinline__ Acc identity() { return lowest<T>(); }
   static __device__ __forceinline__ Acc lift(T x) { return x; }
-  static __device__ __forceinline__ Acc combine(Acc a, Acc b) {
-    // take b if a is NaN, b is larger, or b is the +0 of a +-0 pair
-    return (a != a || b > a || (b == a && !sign_bit(b))) ? b : a;
-  }
+  static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a == b ? bits_and(a, b) : hw_max(a, b); }
   static __device__ __forceinline__ T finish(Acc a) { return a; }
 };
 template <typename T> struct Op<OP_MIN, T, true> {
   using Acc = T;
   static __device__ __forceinline__ Acc identity() { return highest<T>(); }
   static __device__ __forceinline__ Acc lift(T x) { return x; }
-  static __device__ __forceinline__ Acc combine(Acc a, Acc b) {
-    return (a != a || b < a || (b == a && sign_bit(b))) ? b : a;
-  }
+  static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a == b ? bits_or(a, b) : hw_min(a, b); }
   static __device__ __forceinline__ T finish(Acc a) { return a; }
 };
 
@@ -222,4 +228,39 @@ template <typename T> __device__ __forceinline__ T unpack(const U128& u, int q) 
   }
 }
 
+}  // namespace xr
+
+namespace xr {
+// ------------------------------------------------------------ bulk async copy
+// cp.async.bulk (the TMA engine's 1-D copy, SASS UBLKCP) global -> shared,
+// completing on an mbarrier with a transaction byte count.
+__device__ __forceinline__ unsigned smem_addr(const void* p) {
+  return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_addr(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_addr(dst)),
+      "l"(src), "r"(bytes), "r"(smem_addr(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "XR_WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra XR_WAIT_%=;\n}" ::"r"(smem_addr(bar)),
+      "r"(parity)
+      : "memory");
+}
 }  // namespace xr

@@ -13,6 +13,7 @@
 //      adjacent levels are one contiguous level), (3) the remaining pattern is
 //      one of R, KR, RK, KRK, RKR, K.
 #include <algorithm>
+#include <cstdlib>
 
 #include "../../include/xreduce.h"
 #include "xr_internal.h"
@@ -104,9 +105,9 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int64_t NW = kBlock / 32;
     int64_t S = 1;
     const int64_t base = B * tiles;
-    if (base < 2 * target_ctas) {
-      S = cdiv(2 * target_ctas, base);
-      S = std::min<int64_t>(S, std::max<int64_t>(1, R / (NW * kUnroll)));
+    if (base < kUnitsPerCta * target_ctas) {
+      S = cdiv(kUnitsPerCta * target_ctas, base);
+      S = std::min<int64_t>(S, std::max<int64_t>(1, R / (4 * NW * kUnroll)));
       S = std::min<int64_t>(S, 1024);
     }
     if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * NW * kUnroll));
@@ -116,6 +117,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     p->splits = S;
     p->units = B * tiles * S;
     p->group = kBlock;
+    p->sched = true;
     if (S > 1) {
       p->ws_bytes = B * tiles * S * TW * asz;
       p->tickets = B * tiles;
@@ -136,11 +138,19 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
   const int64_t work = C * L;  // elements per output
+  // CTA-wide groups claim units dynamically: over-decompose for tail balance
+  const int64_t want_units = (W == kBlock ? kUnitsPerCta : 2) * resident_groups(W);
   int64_t S = 1;
-  if (O < 2 * resident_groups(W)) {
-    S = cdiv(2 * resident_groups(W), O);
-    S = std::min<int64_t>(S, std::max<int64_t>(1, work / min_unit_elems(W)));
+  if (O < want_units) {
+    S = cdiv(want_units, O);
+    S = std::min<int64_t>(S, std::max<int64_t>(1, work / (4 * min_unit_elems(W))));
   }
+  // long contiguous rows (R, KR): the bulk-copy stream kernel; every unit must
+  // cover at least kStages stages so the producer stays <= 3 units ahead
+  const int64_t stage_elems = kStageBytes / size;
+  const bool stream = C == 1 && row_bytes >= (int64_t)kStages * kStageBytes && std::getenv("XR_NO_BULK") == nullptr;
+  if (stream) S = std::min<int64_t>(S, std::max<int64_t>(1, work / (kStages * stage_elems)));
+  // fp32 '+': per-thread chains <= kChainCap (stream: 16 accumulators per thread)
   if (chain_capped) S = std::max<int64_t>(S, cdiv(work, (int64_t)kChainCap * W * vec * kUnroll));
   if (S > 1 && W < 32) W = 32;  // the gang-tier ticket runs per warp or per CTA
   int64_t Sr, Sc;
@@ -148,8 +158,9 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   else { Sr = C; Sc = std::min<int64_t>(cdiv(S, C), std::max<int64_t>(1, L / vec)); }
   S = Sr * Sc;
 
-  p->kernel = K_SEG;
+  p->kernel = stream ? K_STREAM : K_SEG;
   p->group = W;
+  p->sched = (W == kBlock);
   p->vec = vec;
   p->splits = S;
   p->units = O * S;

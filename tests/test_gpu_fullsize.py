@@ -1,0 +1,148 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration
+bench.py times (same xr_reduce entry point, same plan).  Where the output is
+large, outputs are SAMPLED and the oracle computes each sampled output on its
+own segment (gathered in the paper's k -> j -> i order); single outputs use
+the full oracle or a closed form that holds at any size."""
+import numpy as np
+import pytest
+
+import datagen
+from datagen import recipes
+import oracle
+from gpu_util import TAU, UNIT, check, torch_dt
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+ALL_MASKS = ["g", "w", "v", "gw", "gv", "wv", "gwv"]
+
+
+def gpu_full(op, dtype, dims, levels, x_dev):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    n = xr.xr_out_count(dims, levels)
+    out = torch.empty(n, dtype=x_dev.dtype, device="cuda")
+    st = xr.xr_reduce(op, dtype, dims, levels, x_dev.data_ptr(), out.data_ptr(),
+                      torch.cuda.current_stream().cuda_stream)
+    assert st == 0, xr.xr_strerror(st)
+    return out.cpu().numpy()
+
+
+def sampled_check(op, dtype, dims, levels, x, gpu, nsamples=192, seed=0):
+    """Oracle per sampled output: gather the segment of output o and reduce it."""
+    mask = oracle.mask_of(levels)
+    kept = [d for d in range(3) if not (mask >> d) & 1]
+    X = x.reshape(dims)
+    count = gpu.size
+    rng = np.random.default_rng(seed)
+    outs = np.unique(np.concatenate([[0, count - 1], rng.integers(0, count, nsamples)]))
+    for o in outs:
+        idx = [slice(None)] * 3
+        rem = int(o)
+        for d in reversed(kept):
+            idx[d] = rem % dims[d]
+            rem //= dims[d]
+        seg = np.ascontiguousarray(X[tuple(idx)]).reshape(-1)
+        check(op, dtype, (seg.size, 1, 1), "gwv", gpu[o:o + 1], seg)
+
+
+# ---------------------------------------------------------------- config 2
+@pytest.mark.parametrize("op,dtype,kind", [("+", "fp32", "u01"), ("max", "fp32", "maxmin"),
+                                           ("min", "fp32", "maxmin"), ("+", "int64", "ints"),
+                                           ("max", "int64", "maxmin"), ("min", "int64", "maxmin")])
+def test_cfg2_1d_2e30(op, dtype, kind):
+    import torch
+    n = 1 << 30
+    seed = datagen.case_seed(2, oracle.OPS[op], oracle.DTYPES[dtype], 7)
+    if kind == "ints":
+        x = datagen.uniform_int(seed, n, -(2**31), 2**31 - 1, np.int64)
+    else:
+        x = recipes.make(kind, (n, 1, 1), 7, dtype, seed)
+    xd = torch.from_numpy(x).cuda()
+    g = gpu_full(op, dtype, (n, 1, 1), "gwv", xd)
+    check(op, dtype, (n, 1, 1), "gwv", g, x)
+    if dtype == "int64" and op in ("max", "min"):
+        assert g[0] == (n - 1 if op == "max" else 0)  # P4: a permutation of 0..n-1
+    del xd
+
+
+def test_cfg2_int64_linear_closed_form():
+    """P1 at full size: sum of 0..2^30-1 = 2^59 - 2^29 (no wrap)."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    n = 1 << 30
+    x = torch.arange(n, dtype=torch.int64, device="cuda")
+    assert xr.reduce(x, "+", "gwv", nest=(n, 1, 1)).item() == 2**59 - 2**29
+    assert xr.reduce(x.to(torch.int32), "^", "gwv", nest=(n, 1, 1)).item() == 0  # P3, m%4 == 3
+    assert xr.reduce(torch.ones(n, dtype=torch.float32, device="cuda"), "+", "gwv",
+                     nest=(n, 1, 1)).item() == float(n)  # P2: exact (chains are short)
+
+
+# ---------------------------------------------------------------- config 3
+@pytest.mark.parametrize("kind", ["um11", "intvals"])
+def test_cfg3_rows_and_columns(kind):
+    import torch
+    R = C = 32768
+    x = recipes.make(kind, (R, 1, C), 4, "fp32", 3)
+    xd = torch.from_numpy(x).cuda()
+    rows = gpu_full("+", "fp32", (R, 1, C), "v", xd)       # row-wise (vector level)
+    cols = gpu_full("+", "fp32", (1, R, C), "w", xd)       # column-wise (worker level)
+    cols_g = gpu_full("+", "fp32", (R, 1, C), "g", xd)     # same columns at gang level
+    exact = kind == "intvals"
+    if exact:  # S <= 2^19 per segment: every order is exact -> bit-exact, check all outputs
+        X = x.reshape(R, C).astype(np.int64)
+        assert np.array_equal(rows.astype(np.int64), X.sum(1))
+        assert np.array_equal(cols.astype(np.int64), X.sum(0))
+        assert np.array_equal(cols, cols_g)
+    else:
+        sampled_check("+", "fp32", (R, 1, C), "v", x, rows)
+        sampled_check("+", "fp32", (1, R, C), "w", x, cols)
+        assert np.array_equal(cols.view(np.uint32), cols_g.view(np.uint32))
+
+
+# ---------------------------------------------------------------- config 4
+def test_cfg4_heat_8192_bitwise():
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    n, iters = 8192, 4
+    T0 = oracle.heat_init(n, n)
+    ref_T, ref_res = oracle.heat(n, n, iters, T0)
+    t1 = torch.from_numpy(T0).cuda()
+    t2 = t1.clone()
+    res = torch.zeros(iters, dtype=torch.float64, device="cuda")
+    assert xr.xr_heat_run(n, n, iters, t1.data_ptr(), t2.data_ptr(), res.data_ptr(),
+                          torch.cuda.current_stream().cuda_stream) == 0
+    torch.cuda.synchronize()
+    assert res.cpu().tolist() == ref_res.tolist()
+    final = (t1 if iters % 2 == 0 else t2).cpu().numpy()
+    assert np.array_equal(final.view(np.uint64), ref_T.view(np.uint64))
+
+
+# ---------------------------------------------------------------- config 5
+CFG5_OPS = ["*", "&", "|", "^", "&&", "||"]
+KIND = {"*": "mul", "&": "band", "|": "bor", "^": "bxor", "&&": "land", "||": "lor"}
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("op", CFG5_OPS)
+def test_cfg5_op_type_matrix_512cubed(op, dtype):
+    """Every cell of the 6 ops x 4 dtypes x 7 masks sweep on 512^3; fp bitwise
+    cells must return XR_ERR_UNSUPPORTED (C3)."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    dims = (512, 512, 512)
+    if dtype.startswith("fp") and op in ("&", "|", "^"):
+        x = torch.zeros(8, dtype=torch_dt(dtype), device="cuda")
+        out = torch.zeros(8, dtype=torch_dt(dtype), device="cuda")
+        for lv in ALL_MASKS:
+            assert xr.xr_reduce(op, dtype, dims, lv, x.data_ptr(), out.data_ptr()) == xr.ERR_UNSUPPORTED
+        return
+    for lv in ALL_MASKS:
+        mask = oracle.mask_of(lv)
+        x = recipes.make(KIND[op], dims, mask, dtype, datagen.case_seed(5, oracle.OPS[op],
+                                                                       oracle.DTYPES[dtype], mask))
+        xd = torch.from_numpy(x).cuda()
+        g = gpu_full(op, dtype, dims, lv, xd)
+        if g.size <= 512:
+            check(op, dtype, dims, lv, g, x, exact=(op == "*"))
+        else:
+            sampled_check(op, dtype, dims, lv, x, g, nsamples=96, seed=mask)
+        del xd
