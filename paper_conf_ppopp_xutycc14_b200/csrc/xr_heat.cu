@@ -13,6 +13,8 @@
 // last-CTA tiers of xr_ops.cuh.  Arithmetic uses __dadd_rn/__dmul_rn so no FMA
 // contraction can occur (the paper disables FMA, @35389-35893), which makes
 // the result bit-identical to the oracle.
+#include <cstdlib>
+
 #include "../../include/xreduce.h"
 #include "xr_internal.h"
 #include "xr_ops.cuh"
@@ -144,10 +146,114 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
   }
 }
 
+// Bulk-copy variant (ni even, T1/T2 16-B aligned): the CTA owns a tile of
+// kTileCols columns x kHeatRows rows.  Thread 0 streams the T1 row windows
+// [c0-2, c0+kTileCols+2) of rows j0-1 .. j1 into a ring of kHeatSlots
+// shared-memory slots with cp.async.bulk (completion on per-slot mbarriers),
+// kHeatSlots-2 rows ahead; each thread computes 2 columns of a row from the
+// three slots (up / cur / down), stores them with 16-B streaming stores and
+// folds |T2 - T1| into its private max.  Bytes in flight no longer depend on
+// registers, and every T1 byte is read from HBM once per tile (halo rows and
+// columns are ~3% extra).
+constexpr int kTileCols = 2 * kBlock;          // 512 doubles = 4 KiB per row
+constexpr int kSlotDoubles = kTileCols + 4;    // + 2-column halo on both sides
+constexpr int kHeatSlots = 8;
+
+__global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
+  using O = Op<OP_MAX, double>;
+  __shared__ __align__(128) double slots[kHeatSlots][kSlotDoubles];
+  __shared__ __align__(8) uint64_t full[kHeatSlots];
+  __shared__ double smem[32];
+  __shared__ int s_last;
+  const int tid = threadIdx.x;
+  const int64_t ni = a.ni;
+  const int64_t c0 = (int64_t)blockIdx.x * kTileCols;
+  const int64_t j0 = 1 + (int64_t)blockIdx.y * kHeatRows;
+  const int64_t j1 = min(j0 + kHeatRows, a.nj - 1);  // output rows [j0, j1)
+  const int64_t nrows = j1 - j0 + 2;                 // loaded rows j0-1 .. j1
+  // window of every row: columns [ws, we) placed at slot offset ws - (c0 - 2)
+  const int64_t ws = max(c0 - 2, (int64_t)0), we = min(c0 + kTileCols + 2, ni);
+  const unsigned wbytes = (unsigned)((we - ws) * 8);
+  const int64_t soff = ws - (c0 - 2);
+  double err = 0.0;
+
+  if (j0 < j1) {
+    if (tid == 0) {
+      for (int k = 0; k < kHeatSlots; ++k) mbar_init(&full[k], 1);
+      fence_mbar_init();
+      for (int64_t r = 0; r < min((int64_t)kHeatSlots, nrows); ++r) {
+        mbar_expect_tx(&full[r], wbytes);
+        bulk_g2s(&slots[r][soff], a.T1 + (j0 - 1 + r) * ni + ws, wbytes, &full[r]);
+      }
+    }
+    __syncthreads();
+    mbar_wait(&full[0], 0);  // row j0-1
+    mbar_wait(&full[1], 0);  // row j0
+    const int64_t col = c0 + 2 * tid;  // my two columns: col, col+1
+    const int li = 2 + 2 * tid;        // their slot index
+    const bool i0 = col >= 1 && col <= ni - 2;          // interior columns
+    const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
+    for (int64_t r = 1; r < nrows - 1; ++r) {  // output row j = j0 + r - 1
+      const int64_t rd = r + 1;               // the "down" row
+      mbar_wait(&full[rd % kHeatSlots], (unsigned)((rd / kHeatSlots) & 1));
+      if (i0 || i1) {
+        const double* up = slots[(r - 1) % kHeatSlots];
+        const double* cur = slots[r % kHeatSlots];
+        const double* dn = slots[rd % kHeatSlots];
+        const double2 u2 = *reinterpret_cast<const double2*>(up + li);
+        const double2 c2 = *reinterpret_cast<const double2*>(cur + li);
+        const double2 d2 = *reinterpret_cast<const double2*>(dn + li);
+        const double l = cur[li - 1], rr = cur[li + 2];
+        const double n0 = stencil(u2.x, d2.x, l, c2.y);
+        const double n1 = stencil(u2.y, d2.y, c2.x, rr);
+        double* dst = a.T2 + (j0 + r - 1) * ni + col;
+        if (i0 && i1) {
+          __stcs(reinterpret_cast<double2*>(dst), make_double2(n0, n1));
+        } else if (i0) {
+          __stcs(dst, n0);
+        } else {
+          __stcs(dst + 1, n1);
+        }
+        if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
+        if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
+      }
+      __syncthreads();  // row r-1 is dead: refill its slot kHeatSlots rows ahead
+      if (tid == 0) {
+        const int64_t nr = r - 1 + kHeatSlots;
+        if (nr < nrows) {
+          const int slot = (int)(nr % kHeatSlots);
+          mbar_expect_tx(&full[slot], wbytes);
+          bulk_g2s(&slots[slot][soff], a.T1 + (j0 - 1 + nr) * ni + ws, wbytes, &full[slot]);
+        }
+      }
+    }
+  }
+  err = block_reduce<OP_MAX, double, kBlock>(err, smem);
+  const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
+  if (tid == 0) {
+    a.partials[cta] = err;
+    __threadfence();
+    const unsigned t = atomicAdd(a.tickets, 1u);
+    s_last = (t == (unsigned)(a.ntiles - 1));
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    double w = 0.0;
+    for (int64_t k = tid; k < a.ntiles; k += kBlock) w = O::combine(w, ld_partial(a.partials + k));
+    w = block_reduce<OP_MAX, double, kBlock>(w, smem);
+    if (tid == 0) {
+      *a.residual = w;
+      *a.tickets = 0u;
+    }
+  }
+}
+
 static int heat_launch(int64_t nj, int64_t ni, const double* T1, double* T2, double* residual,
                        cudaStream_t s) {
   const bool v2 = (ni % 2 == 0) && ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
-  const int strip = 32 * (v2 ? 2 : 1) * (kBlock / 32);
+  const bool bulk = v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr;
+  const int strip = bulk ? kTileCols : 32 * (v2 ? 2 : 1) * (kBlock / 32);
   const int64_t gx = (ni + strip - 1) / strip;
   const int64_t gy = nj > 2 ? (nj - 2 + kHeatRows - 1) / kHeatRows : 1;
   if (gy > 65535) return XR_ERR_INVALID;
@@ -160,7 +266,8 @@ static int heat_launch(int64_t nj, int64_t ni, const double* T1, double* T2, dou
   a.partials = static_cast<double*>(partials);
   a.tickets = tickets;
   dim3 grid((unsigned)gx, (unsigned)gy);
-  if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
+  if (bulk) heat_bulk_kernel<<<grid, kBlock, 0, s>>>(a);
+  else if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
   else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);
   count_launch();
   if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }

@@ -82,11 +82,17 @@ __device__ __forceinline__ typename Op<OP, T>::Acc seg_unit(const SegArgs& a, in
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
-  const int64_t S = a.Sr * a.Sc;
-  const int64_t o = u / S, s = u - o * S;
-  const int64_t sr = s / a.Sc, sc = s - sr * a.Sc;
-  const int64_t r0 = split_lo(a.C, a.Sr, sr), r1 = split_lo(a.C, a.Sr, sr + 1);
-  const int64_t c0 = split_lo_vec(a.L, a.Sc, sc, VEC), c1 = split_lo_vec(a.L, a.Sc, sc + 1, VEC);
+  int64_t o, r0, r1, c0, c1;
+  if (a.Sr == 1 && a.Sc == 1) {  // unsplit: no 64-bit divisions on the per-row path
+    o = u; r0 = 0; r1 = a.C; c0 = 0; c1 = a.L;
+  } else {
+    const int64_t S = a.Sr * a.Sc;
+    o = u / S;
+    const int64_t s = u - o * S;
+    const int64_t sr = s / a.Sc, sc = s - sr * a.Sc;
+    r0 = split_lo(a.C, a.Sr, sr); r1 = split_lo(a.C, a.Sr, sr + 1);
+    c0 = split_lo_vec(a.L, a.Sc, sc, VEC); c1 = split_lo_vec(a.L, a.Sc, sc + 1, VEC);
+  }
   Acc acc[U][VEC];
 #pragma unroll
   for (int k = 0; k < U; ++k)
@@ -324,18 +330,23 @@ __global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
   }
   __syncthreads();
 
+  // One output (R shape): every unit's partial goes to partials[u] with no
+  // per-unit fence or ticket; each CTA takes ONE ticket at exit and the last
+  // CTA combines the S unit partials in unit order -- deterministic although
+  // units are claimed dynamically.  Several outputs: per-unit ticket per output.
+  const bool whole = (a.O == 1);
   int seq = 0;
   int64_t g = 0;  // consumer's global chunk index (stage = g % NS, phase parity = (g / NS) & 1)
+  Acc acc[PER][VEC];
+#pragma unroll
+  for (int j = 0; j < PER; ++j)
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
   while (true) {
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
     const StreamGeom geo = stream_geom<T>(a, u);
     const T* row = static_cast<const T*>(geo.row);
-    Acc acc[PER][VEC];
-#pragma unroll
-    for (int j = 0; j < PER; ++j)
-#pragma unroll
-      for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
     if (tid < geo.head) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(row + tid)));
     if (tid < geo.tail)
       acc[0][VEC - 1] = O::combine(acc[0][VEC - 1], O::lift(ld_scalar(row + geo.head + geo.nbody + tid)));
@@ -359,9 +370,15 @@ __global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
       if (tid == 0) p_issue();    // refill it NS chunks ahead
     }
     Acc v = fold_acc<OP, T, PER, VEC>(acc);
+#pragma unroll
+    for (int j = 0; j < PER; ++j)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
     v = block_reduce<OP, T, BLOCK>(v, smem);
     const int64_t o = geo.o;
-    if (S == 1) {
+    if (whole) {
+      if (tid == 0) partials[u] = v;
+    } else if (S == 1) {
       if (tid == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
     } else {
       if (tid == 0) {
@@ -383,6 +400,23 @@ __global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
     }
     __syncthreads();
     ++seq;
+  }
+  if (whole) {  // a4: one ticket per CTA; the last CTA combines the S unit partials
+    if (tid == 0) {
+      __threadfence();
+      const unsigned t = atomicAdd(&a.tickets[0], 1u);
+      s_last = (t == gridDim.x - 1u);
+    }
+    __syncthreads();
+    if (s_last) {
+      __threadfence();
+      Acc w = fold_partials<OP, T>(partials, S, tid, BLOCK);
+      w = block_reduce<OP, T, BLOCK>(w, smem);
+      if (tid == 0) {
+        out[0] = merge_init<OP, T>(w, out, 0, a.init_from_out);
+        a.tickets[0] = 0u;
+      }
+    }
   }
   sched_exit(a.sched);
 }

@@ -149,7 +149,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // cover at least kStages stages so the producer stays <= 3 units ahead
   const int64_t stage_elems = kStageBytes / size;
   const bool stream = C == 1 && row_bytes >= (int64_t)kStages * kStageBytes && std::getenv("XR_NO_BULK") == nullptr;
-  if (stream) S = std::min<int64_t>(S, std::max<int64_t>(1, work / (kStages * stage_elems)));
+  if (stream) {
+    const int64_t min_stages = O == 1 ? kStages : 4 * kStages;  // several outputs: amortise the epilogue
+    S = std::min<int64_t>(S, std::max<int64_t>(1, work / (min_stages * stage_elems)));
+  }
   // fp32 '+': per-thread chains <= kChainCap (stream: 16 accumulators per thread)
   if (chain_capped) S = std::max<int64_t>(S, cdiv(work, (int64_t)kChainCap * W * vec * kUnroll));
   if (S > 1 && W < 32) W = 32;  // the gang-tier ticket runs per warp or per CTA
@@ -167,6 +170,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   if (S > 1) {
     p->ws_bytes = O * S * asz;
     p->tickets = O;
+  }
+  if (stream && O == 1) {  // unit partials + one CTA-exit ticket, also when S == 1
+    p->ws_bytes = std::max<int64_t>(S, 1) * asz;
+    p->tickets = 1;
   }
   SegArgs& s = p->seg;
   s.O = O; s.C = C; s.L = L; s.rowStride = rowStride; s.oStride = oStride;

@@ -24,3 +24,12 @@ for f in [f"gpurun_out/shapes_{tag}.jsonl", f"gpurun_out/cfg5_{tag}.jsonl"]:
 b = open(f"gpurun_out/bench_{tag}.json").read().strip()
 print(b[:600])
 PY
+if [ "${NCU:-0}" = "1" ]; then
+  mkdir -p gpurun_out/ncu
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ncu/launches_$TAG.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline --e2e-steps 0 > gpurun_out/ncu/launches_$TAG.log 2>&1
+  for c in "stream_kernel cfg2-f32-sum fp32sum" "col_kernel cfg3-col cfg3col" "stream_kernel cfg3-row cfg3row" "heat cfg4-heat heat" "seg_kernel cfg5-land-int32-v cfg5v"; do
+    set -- $c
+    timeout 600 ncu --set full --clock-control none --import-source on -k regex:$1 -s 3 -c 1 -o gpurun_out/ncu/$3_$TAG -f python tools/kdriver.py $2 --reps 1 > gpurun_out/ncu/$3_$TAG.log 2>&1
+  done
+  ls gpurun_out/ncu
+fi
