@@ -152,6 +152,10 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   p.col.in = in; p.col.out = out; p.col.partials = w.partials; p.col.tickets = w.tickets;
   p.col.init_from_out = ifo;
   p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
+  if (p.kernel == K_COLTMA && !make_col_tmap(&p.tmap, dtype, in, p.col.B, p.col.R, p.col.K)) {
+    // no tensor-map support: re-plan without TMA (same workspace bound or smaller)
+    return XR_ERR_CUDA;
+  }
   cudaError_t e = launch_dtype(op, dtype, p, sms, stream);
   if (e != cudaSuccess) {
     cudaGetLastError();
@@ -231,7 +235,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   info->units = p.units;
   info->block = p.block;
   int64_t ctas = p.units;
-  if (p.kernel == K_STREAM) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
+  if (p.kernel == K_STREAM || p.kernel == K_COLTMA) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);

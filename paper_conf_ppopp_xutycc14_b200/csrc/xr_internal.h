@@ -2,6 +2,7 @@
 // translation units (never installed, never seen by the oracle).
 #pragma once
 #include <cstdint>
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 namespace xr {
@@ -12,7 +13,7 @@ constexpr int kChainCap = 4096; // max sequential fp32 '+' chain per accumulator
 constexpr int kTargetCtasPerSm = 8;  // 2048 threads/SM at 256 threads/CTA
 constexpr int kUnitsPerCta = 8;      // dynamic units per resident CTA (tail balance)
 
-enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5 };
+enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6 };
 
 constexpr int kStages = 4;          // bulk-copy ring depth (stream kernel)
 constexpr int kStageBytes = 16384;  // bytes per stage
@@ -41,8 +42,11 @@ struct ColArgs {
   int64_t B, R, K;
   int64_t tiles, S;
   int64_t units;       // B * tiles * S
+  int64_t G2;          // coltma: groups of kGroupFold unit partials per tile (two-level gang tier)
   int init_from_out;
 };
+
+constexpr int kGroupFold = 64;  // unit partials folded per group by the group's last CTA
 
 // Elementwise: out[o] = init (+) in[o] (ident) or out[o] = init (fill).
 struct EltArgs {
@@ -67,6 +71,7 @@ struct Plan {
   bool sched = false;   // CTA-wide units are claimed dynamically (2 extra counters)
   SegArgs seg{};
   ColArgs col{};
+  CUtensorMap tmap{};   // K_COLTMA: 3-D map over (K, R, B), built at launch
   EltArgs elt{};
 };
 
@@ -91,6 +96,10 @@ cudaError_t gather_i32(int op, const void* g, int nranks, int64_t n, void* out, 
 cudaError_t gather_i64(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
 cudaError_t gather_f32(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
 cudaError_t gather_f64(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+
+// Encode the K_COLTMA tensor map for `in` (false if the driver entry point or
+// the encode fails; the caller then falls back to the register column kernel).
+bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K);
 
 // Grid for `units` work items given the device's resident-CTA budget.
 int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm);

@@ -6,6 +6,8 @@
 // another kernel ... is launched" (PAPER.md @24887-25280, 3.1.3) and the RMP
 // global buffer + second kernel (@29217-29414, @31388-31587).
 #pragma once
+#include <cuda.h>
+
 #include <algorithm>
 
 #include "xr_internal.h"
@@ -276,7 +278,7 @@ __global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
   constexpr int PER = STAGE / (16 * BLOCK);  // 16-B vectors per thread per stage
   constexpr int RING = 8;                    // published unit ids (producer <= 3 units ahead)
   static_assert(PER >= 1 && STAGE % (16 * BLOCK) == 0, "stage geometry");
-  extern __shared__ __align__(128) unsigned char stage_mem[];  // NS * STAGE
+  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE
   __shared__ __align__(8) uint64_t full[NS];
   __shared__ long long s_units[RING];
   __shared__ Acc smem[32];
@@ -504,9 +506,9 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
     } else {  // a4: gang tier per column tile
       Acc* P = partials + (b * a.tiles + tile) * a.S * TW;
       if (t < TW) P[s * TW + t] = v;
-      __threadfence();
-      __syncthreads();
+      __syncthreads();  // the CTA's partial stores happen-before thread 0's fence (cumulative)
       if (t == 0) {
+        __threadfence();
         const unsigned tk = atomicAdd(&a.tickets[b * a.tiles + tile], 1u);
         s_last = (tk == (unsigned)(a.S - 1));
       }
@@ -546,6 +548,209 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
     __syncthreads();
     u = s_unit[par];
     par ^= 1;
+  }
+  sched_exit(a.sched);
+}
+
+// ------------------------------------------------------------- col TMA kernel
+// RK / KRK with 16-B aligned rows of >= 1 KiB: a 3-D TMA tensor map over
+// (K, R, B) loads boxes of 1 KiB x kColBoxRows rows into the shared-memory
+// ring (cp.async.bulk.tensor, SASS UTMALDG), thread 0 producing NS boxes ahead
+// across unit boundaries.  Threads own a 16-B column group and a row phase;
+// the worker tier folds the row phases per column in shared memory; the gang
+// tier is the per-tile ticket of col_kernel.  OOB rows/columns of a box are
+// skipped by the consumers, so the fill value never matters.
+template <int OP, typename T, int BLOCK, int NS>
+__global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int TW = 1024 / (int)sizeof(T);  // box columns
+  constexpr int BR = kStageBytes / 1024;     // box rows
+  constexpr int G = TW / VEC;                // 16-B column groups per row
+  constexpr int NPH = BLOCK / G;             // row phases
+  constexpr int PH2 = BLOCK / TW;            // threads per column in the tile combine
+  constexpr int RING = 8;
+  constexpr int AV = 16 / (int)sizeof(Acc);  // partials per 16-B load in the folds
+  constexpr int NPA = BLOCK / (TW / AV);     // row phases of the folds
+  constexpr int NRED = NPH > NPA ? NPH : NPA;
+  static_assert(NPH >= 1 && PH2 >= 1 && NPA >= 1 && BR % NPH == 0, "geometry");
+  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * kStageBytes
+  __shared__ __align__(8) uint64_t full[NS];
+  __shared__ long long s_units[RING];
+  __shared__ __align__(16) Acc red[NRED][TW];
+  __shared__ int s_last;
+  const int tid = threadIdx.x, grp = tid % G, ph = tid / G;
+  T* out = static_cast<T*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  const int64_t per_b = a.tiles * a.S;
+
+  // ---- producer (thread 0)
+  long long p_unit = 0, p_next = 0;
+  int64_t p_k = 0, p_nk = 0, g_issue = 0, p_b = 0, p_tile = 0, p_r0 = 0;
+  int p_seq = 0;
+  auto p_start = [&](long long u) {
+    p_unit = u;
+    s_units[p_seq & (RING - 1)] = u < a.units ? u : -1;
+    ++p_seq;
+    p_k = 0;
+    p_nk = 0;
+    if (u < a.units) {
+      p_b = u / per_b;
+      const int64_t rem = u - p_b * per_b;
+      p_tile = rem / a.S;
+      const int64_t s = rem - p_tile * a.S;
+      p_r0 = split_lo(a.R, a.S, s);
+      p_nk = (split_lo(a.R, a.S, s + 1) - p_r0 + BR - 1) / BR;
+    }
+  };
+  auto p_issue = [&]() {
+    while (p_unit < a.units && p_k == p_nk) {
+      const long long nu = p_next;
+      p_next = (long long)atomicAdd(a.sched, 1ull);
+      p_start(nu);
+    }
+    if (p_unit >= a.units) return;
+    const int slot = (int)(g_issue % NS);
+    mbar_expect_tx(&full[slot], (unsigned)kStageBytes);
+    tma_load_3d(stage_mem + slot * kStageBytes, &tmap, (int)(p_tile * TW), (int)(p_r0 + p_k * BR), (int)p_b,
+                &full[slot]);
+    ++p_k;
+    ++g_issue;
+  };
+  if (tid == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
+#pragma unroll
+    for (int k = 0; k < NS; ++k) mbar_init(&full[k], 1);
+    fence_mbar_init();
+    const long long u0 = (long long)atomicAdd(a.sched, 1ull);
+    p_next = (long long)atomicAdd(a.sched, 1ull);
+    p_start(u0);
+    for (int k = 0; k < NS; ++k) p_issue();
+  }
+  __syncthreads();
+
+  int seq = 0;
+  int64_t g = 0;
+  while (true) {
+    const long long u = s_units[seq & (RING - 1)];
+    if (u < 0) break;
+    const int64_t b = u / per_b, rem = u - b * per_b;
+    const int64_t tile = rem / a.S, s = rem - tile * a.S;
+    const int64_t r0 = split_lo(a.R, a.S, s), r1 = split_lo(a.R, a.S, s + 1);
+    const int64_t nk = (r1 - r0 + BR - 1) / BR;
+    const bool col_ok = tile * TW + (int64_t)grp * VEC < a.K;  // K % VEC == 0: whole vectors
+    Acc acc[2][VEC];
+#pragma unroll
+    for (int j = 0; j < 2; ++j)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
+    for (int64_t k = 0; k < nk; ++k, ++g) {
+      const int slot = (int)(g % NS);
+      mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      const unsigned char* st = stage_mem + slot * kStageBytes;
+      const int64_t rbase = r0 + k * BR;
+#pragma unroll
+      for (int i = 0; i < BR / NPH; ++i) {
+        const int row = ph + i * NPH;
+        if (col_ok && rbase + row < r1) {
+          const U128 x = *reinterpret_cast<const U128*>(st + row * 1024 + grp * 16);
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
+        }
+      }
+      __syncthreads();
+      if (tid == 0) p_issue();
+    }
+    // a3: fold the row phases per column
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) red[ph][grp * VEC + q] = O::combine(acc[0][q], acc[1][q]);
+    __syncthreads();
+    const int64_t oc = tile * TW + tid;  // output column of thread tid (< TW)
+    Acc v = O::identity();
+    if (tid < TW) {
+#pragma unroll
+      for (int p2 = 0; p2 < NPH; ++p2) v = O::combine(v, red[p2][tid]);
+    }
+    if (a.S == 1) {
+      if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(v, out, b * a.K + oc, a.init_from_out);
+    } else {
+      // a4, two levels: unit partial -> group of kGroupFold (its last CTA folds
+      // the group in unit order) -> tile (the last group folds the G2 group
+      // partials).  Keeps every fold short although S can be ~1000.
+      const int64_t tid_tile = b * a.tiles + tile;
+      Acc* P1 = partials + tid_tile * a.S * TW;                                  // [S][TW]
+      Acc* P2 = partials + a.B * a.tiles * a.S * TW + tid_tile * a.G2 * TW;      // [G2][TW]
+      unsigned* gt = a.tickets + tid_tile * a.G2;                                // group tickets
+      unsigned* tt = a.tickets + a.B * a.tiles * a.G2 + tid_tile;                // tile ticket
+      const int64_t grp_i = s / kGroupFold;
+      const int64_t g0 = grp_i * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
+      // fold rows [0, n) of a [n][TW] partial block into column tid (< TW):
+      // 16-B L2 loads, NPA row phases x (TW/AV) column groups, 4 rows in flight
+      auto fold_rows = [&](const Acc* base, int64_t n) -> Acc {
+        const int cg = tid % (TW / AV), q2 = tid / (TW / AV);
+        Acc w[AV];
+#pragma unroll
+        for (int q = 0; q < AV; ++q) w[q] = O::identity();
+        int64_t r = q2;
+        for (; r + 3 * NPA < n; r += 4 * NPA) {
+          uint4 y[4];
+#pragma unroll
+          for (int k = 0; k < 4; ++k) y[k] = __ldcg(reinterpret_cast<const uint4*>(base + (r + k * NPA) * TW + cg * AV));
+#pragma unroll
+          for (int k = 0; k < 4; ++k)
+#pragma unroll
+            for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y[k])[q]);
+        }
+        for (; r < n; r += NPA) {
+          const uint4 y = __ldcg(reinterpret_cast<const uint4*>(base + r * TW + cg * AV));
+#pragma unroll
+          for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y)[q]);
+        }
+#pragma unroll
+        for (int q = 0; q < AV; ++q) red[q2][cg * AV + q] = w[q];
+        __syncthreads();
+        Acc z = O::identity();
+        if (tid < TW) {
+#pragma unroll
+          for (int p2 = 0; p2 < NPA; ++p2) z = O::combine(z, red[p2][tid]);
+        }
+        return z;
+      };
+      if (tid < TW) P1[s * TW + tid] = v;
+      __syncthreads();  // partial stores happen-before thread 0's (cumulative) fence
+      if (tid == 0) {
+        __threadfence();
+        const unsigned tk = atomicAdd(&gt[grp_i], 1u);
+        s_last = (tk == (unsigned)(gsz - 1));
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        const Acc w = fold_rows(P1 + g0 * TW, gsz);
+        if (tid == 0) gt[grp_i] = 0u;
+        if (a.G2 == 1) {
+          if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(w, out, b * a.K + oc, a.init_from_out);
+        } else {
+          if (tid < TW) P2[grp_i * TW + tid] = w;
+          __syncthreads();
+          if (tid == 0) {
+            __threadfence();
+            const unsigned tk = atomicAdd(tt, 1u);
+            s_last = (tk == (unsigned)(a.G2 - 1));
+          }
+          __syncthreads();
+          if (s_last) {
+            __threadfence();
+            const Acc z = fold_rows(P2, a.G2);
+            if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(z, out, b * a.K + oc, a.init_from_out);
+            if (tid == 0) *tt = 0u;
+          }
+        }
+      }
+    }
+    __syncthreads();
+    ++seq;
   }
   sched_exit(a.sched);
 }
@@ -628,6 +833,18 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
         return n;
       }();
       kern<<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, dyn, s>>>(p.seg);
+      break;
+    }
+    case K_COLTMA: {
+      auto kern = coltma_kernel<OP, T, kBlock, kStages>;
+      constexpr int dyn = kStages * kStageBytes;
+      static int occ = [&] {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        return n;
+      }();
+      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, dyn, s>>>(p.tmap, p.col);
       break;
     }
     case K_COL: {

@@ -100,6 +100,36 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     else { B = run_n[0]; R = run_n[1]; K = run_n[2]; p->shape = XR_SHAPE_KRK; }
     const bool aligned = ((K * size) % 16 == 0) && (in_addr % 16 == 0);
     const int cv = aligned ? vec : 1;
+    // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
+    if (aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
+        B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {
+      const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
+      const int64_t tiles = cdiv(K, TWt);
+      // ~8 units per resident CTA (3 per SM): a CTA streams ~16.5 GB/s, so the
+      // tail is about one unit (r01i: 4 per CTA left SMs idle 25% of the time),
+      // while each unit still amortises its epilogue (r01j: 16 per CTA too many)
+      const int64_t target = 8 * (int64_t)std::max(num_sms, 1) * 3;
+      int64_t S = cdiv(target, B * tiles);
+      S = std::min<int64_t>(S, std::max<int64_t>(1, R / (kStages * BR)));  // >= kStages boxes per unit
+
+      if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * 8));
+      S = std::max<int64_t>(1, std::min<int64_t>(S, R));
+      p->kernel = K_COLTMA;
+      p->vec = vec;
+      p->splits = S;
+      p->units = B * tiles * S;
+      p->group = kBlock;
+      p->sched = true;
+      // two-level gang tier: groups of kGroupFold unit partials, then the groups
+      const int64_t G2 = cdiv(S, kGroupFold);
+      if (S > 1) {
+        p->ws_bytes = B * tiles * (S + G2) * TWt * asz;
+        p->tickets = B * tiles * (G2 + 1);
+      }
+      ColArgs& c = p->col;
+      c.B = B; c.R = R; c.K = K; c.tiles = tiles; c.S = S; c.units = p->units; c.G2 = G2;
+      return;
+    }
     const int64_t TW = 32 * cv;
     const int64_t tiles = cdiv(K, TW);
     const int64_t NW = kBlock / 32;
@@ -108,7 +138,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     if (base < kUnitsPerCta * target_ctas) {
       S = cdiv(kUnitsPerCta * target_ctas, base);
       S = std::min<int64_t>(S, std::max<int64_t>(1, R / (4 * NW * kUnroll)));
-      S = std::min<int64_t>(S, 1024);
+      S = std::min<int64_t>(S, 128);  // the last CTA of a tile folds S rows (8 warps x 4 loads)
     }
     if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * NW * kUnroll));
     S = std::max<int64_t>(1, std::min<int64_t>(S, R));

@@ -108,7 +108,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     shape, cd = SHAPE_TABLE[levels]
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
-    assert p["kernel"] in (("col",) if shape in ("RK", "KRK") else ("seg", "stream"))
+    assert p["kernel"] in (("col", "coltma") if shape in ("RK", "KRK") else ("seg", "stream"))
 
 
 def test_plan_canonical_cfg2_cfg3_cfg5(xr):
@@ -116,6 +116,7 @@ def test_plan_canonical_cfg2_cfg3_cfg5(xr):
     assert xr.xr_plan_describe("+", "fp32", (32768, 1, 32768), "v", 256)["cdims"] == [32768, 32768, 0]
     c = xr.xr_plan_describe("+", "fp32", (1, 32768, 32768), "w", 256)
     assert c["shape"] == "RK" and c["cdims"] == [32768, 32768, 0] and c["vec"] == 4
+    assert c["kernel"] == "coltma"
     # {1,R,C}+W and {R,1,C}+G run the same column plan (a0)
     c2 = xr.xr_plan_describe("+", "fp32", (32768, 1, 32768), "g", 256)
     assert {k: c[k] for k in ("shape", "cdims", "splits", "units")} == \
@@ -152,9 +153,9 @@ def test_plan_fp32_chain_cap(xr, case):
         c = p["cdims"]
         work = {"R": c[0], "KR": c[1], "RKR": c[0] * c[2]}[p["shape"]]
         per_acc = work / p["splits"] / (p["group"] * p["vec"] * 4)
-    else:
+    else:  # col: 8 warps x 4 rows in flight; coltma: 4 row phases x 2 accumulators
         R = p["cdims"][0] if p["shape"] == "RK" else p["cdims"][1]
-        per_acc = R / p["splits"] / (8 * 4)
+        per_acc = R / p["splits"] / (8 * 4 if p["kernel"] == "col" else 8)
     assert per_acc <= 4096 + 1
 
 
