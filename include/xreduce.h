@@ -39,6 +39,9 @@ extern "C" {
 /* Compatible with cudaStream_t (both are `struct CUstream_st *`). */
 typedef struct CUstream_st* xr_stream_t;
 
+/* Opaque NCCL communicator of the multi-GPU entry points (xr_comm_init). */
+typedef struct xr_comm_s* xr_comm_t;
+
 /* Operators (reading C1: the OpenACC C set; the paper evaluates + and *
  * (@37852-37985) and max (@37985, Fig 13a) and claims "all reduction
  * operator types" (@6300-6414)). */
@@ -186,6 +189,27 @@ int xr_heat_step(int64_t nj, int64_t ni, const double* T1, double* T2, double* r
 int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,
                 double* residuals, xr_stream_t stream);
 
+/* Gang-row sharded heat (config 4 on several GPUs).  Rank r of
+ * nranks owns global rows [r*n_local, (r+1)*n_local) of the
+ * (nranks*n_local) x ni grid, stored in a DEVICE buffer of (n_local+2) x ni
+ * fp64: local row 0 = global row r*n_local-1 and local row n_local+1 = global
+ * row (r+1)*n_local are halos (unused at the global boundary).  Both buffers
+ * must start with the initial field AND the neighbours' halo rows.  One step =
+ * the fused sweep of the owned interior rows, then the halo rows of T2 are
+ * exchanged with grouped ncclSend/ncclRecv and the residual is combined with
+ * ncclAllReduce(max) of one fp64 into *residual (DEVICE) on every rank.  The
+ * results are bit-identical to xr_heat_step on the whole grid. */
+int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* T2,
+                         double* residual, xr_comm_t comm, xr_stream_t stream);
+/* iters steps swapping T1/T2 (residuals: DEVICE, iters fp64). */
+int xr_heat_run_sharded(int64_t n_local, int64_t ni, int64_t iters, double* T1, double* T2,
+                        double* residuals, xr_comm_t comm, xr_stream_t stream);
+/* Single-device simulation of the same protocol over nranks slabs (halo
+ * exchange by device copies, residual by the fixed-order max combine). */
+int xr_heat_run_sharded_sim(int64_t n_local, int64_t ni, int64_t iters, int nranks,
+                            double* const* T1s, double* const* T2s, double* residuals,
+                            xr_stream_t stream);
+
 /* ------------------------------------------------- multi-GPU (gang shards) */
 
 /* Sharding along the gang level: rank r owns the contiguous
@@ -217,8 +241,6 @@ typedef struct {
 /* Host-only: the exchange xr_reduce_sharded performs for this rank. */
 int xr_shard_plan(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
                   int nranks, int rank, xr_shard_info* info);
-
-typedef struct xr_comm_s* xr_comm_t;
 
 /* NCCL unique id (128 bytes) on rank 0; broadcast it out of band
  * (torch.distributed in the Python binding). */

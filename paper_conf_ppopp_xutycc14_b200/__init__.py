@@ -4,7 +4,7 @@ Thin ctypes binding over ``libxreduce.so`` (include/xreduce.h).  Argument
 marshalling only: every step of the reduction runs in the library's CUDA
 kernels.  PyTorch is used for device memory, streams and process groups.
 There is NO CPU fallback: if the shared library is missing this import fails
-loudly (build it with ``python -m paper_conf_ppopp_xutycc14_b200._build`` or
+loudly (build it with ``python tools/build_native.py`` or
 ``__graft_entry__.build()``).
 
 Paper: Xu, Tian, Yan, Chandrasekaran, Chapman, "Reduction Operations in
@@ -20,7 +20,7 @@ LIB_PATH = os.path.join(_HERE, "libxreduce.so")
 if not os.path.exists(LIB_PATH):
     raise ImportError(
         f"xreduce: {LIB_PATH} is missing -- build the CUDA library first "
-        "(python -m paper_conf_ppopp_xutycc14_b200._build); there is no CPU fallback")
+        "(python tools/build_native.py); there is no CPU fallback")
 _lib = ctypes.CDLL(LIB_PATH)
 
 # ---- codes (include/xreduce.h)
@@ -91,6 +91,10 @@ _SIGS = {
     "xr_comm_destroy": (_c, [_vp]),
     "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
+    "xr_heat_step_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
+    "xr_heat_run_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
+    "xr_heat_run_sharded_sim": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _c, ctypes.POINTER(_vp),
+                                     ctypes.POINTER(_vp), _vp, _vp]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -187,6 +191,17 @@ def xr_reduce_sharded_sim(op, dtype, local_dims, level_mask, shard_ptrs, out_ptr
     arr = (_vp * len(shard_ptrs))(*shard_ptrs)
     return _lib.xr_reduce_sharded_sim(_op(op), _dt(dtype), _dims(local_dims), mask_of(level_mask),
                                       arr, len(shard_ptrs), out_ptr, stream or None)
+
+
+def xr_heat_run_sharded_sim(n_local, ni, iters, t1_ptrs, t2_ptrs, residuals_ptr, stream: int = 0) -> int:
+    a = (_vp * len(t1_ptrs))(*t1_ptrs)
+    b = (_vp * len(t2_ptrs))(*t2_ptrs)
+    return _lib.xr_heat_run_sharded_sim(n_local, ni, iters, len(t1_ptrs), a, b, residuals_ptr, stream or None)
+
+
+def xr_heat_run_sharded(n_local, ni, iters, t1_ptr, t2_ptr, residuals_ptr, comm, stream: int = 0) -> int:
+    return _lib.xr_heat_run_sharded(n_local, ni, iters, t1_ptr, t2_ptr, residuals_ptr, comm.handle,
+                                    stream or None)
 
 
 # ---------------------------------------------------------------- torch-facing helpers

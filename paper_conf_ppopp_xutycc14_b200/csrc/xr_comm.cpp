@@ -17,6 +17,9 @@ namespace xr {
 int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask, const void* in, void* out,
                           cudaStream_t s);
 cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
+int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* je);
+int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
+                   double* residual, cudaStream_t s);
 }  // namespace xr
 
 struct xr_comm_s {
@@ -119,6 +122,46 @@ int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned l
     // in place: rank r's segment already sits at out + r*local_count
     if (ncclAllGather(mine, out, (size_t)info.local_count, nccl_type(dtype), comm->nccl, s) != ncclSuccess)
       return XR_ERR_NCCL;
+  }
+  return XR_OK;
+}
+
+int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* T2, double* residual,
+                         xr_comm_t comm, xr_stream_t stream) {
+  if (!comm || !residual || n_local < 1 || ni < 0 || !T1 || !T2) return XR_ERR_INVALID;
+  cudaStream_t s = (cudaStream_t)stream;
+  int64_t jb, je;
+  int st = heat_slab_rows(n_local, comm->nranks, comm->rank, &jb, &je);
+  if (st) return st;
+  if ((st = heat_step_rows(n_local + 2, ni, jb, je, T1, T2, residual, s))) return st;
+  if (comm->nranks == 1) return XR_OK;
+  // halo rows of the new field: my first owned row goes up, my last goes down
+  const int r = comm->rank;
+  if (ncclGroupStart() != ncclSuccess) return XR_ERR_NCCL;
+  if (r > 0) {
+    ncclSend(T2 + ni, (size_t)ni, ncclFloat64, r - 1, comm->nccl, s);
+    ncclRecv(T2, (size_t)ni, ncclFloat64, r - 1, comm->nccl, s);
+  }
+  if (r < comm->nranks - 1) {
+    ncclSend(T2 + n_local * ni, (size_t)ni, ncclFloat64, r + 1, comm->nccl, s);
+    ncclRecv(T2 + (n_local + 1) * ni, (size_t)ni, ncclFloat64, r + 1, comm->nccl, s);
+  }
+  if (ncclGroupEnd() != ncclSuccess) return XR_ERR_NCCL;
+  if (ncclAllReduce(residual, residual, 1, ncclFloat64, ncclMax, comm->nccl, s) != ncclSuccess) return XR_ERR_NCCL;
+  return XR_OK;
+}
+
+int xr_heat_run_sharded(int64_t n_local, int64_t ni, int64_t iters, double* T1, double* T2, double* residuals,
+                        xr_comm_t comm, xr_stream_t stream) {
+  if (iters < 0 || (iters > 0 && !residuals)) return XR_ERR_INVALID;
+  double* a = T1;
+  double* b = T2;
+  for (int64_t it = 0; it < iters; ++it) {
+    int st = xr_heat_step_sharded(n_local, ni, a, b, residuals + it, comm, stream);
+    if (st) return st;
+    double* t = a;
+    a = b;
+    b = t;
   }
   return XR_OK;
 }

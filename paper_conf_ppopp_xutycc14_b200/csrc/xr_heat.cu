@@ -14,6 +14,8 @@
 // contraction can occur (the paper disables FMA, @35389-35893), which makes
 // the result bit-identical to the oracle.
 #include <cstdlib>
+#include <utility>
+#include <vector>
 
 #include "../../include/xreduce.h"
 #include "xr_internal.h"
@@ -33,6 +35,7 @@ struct HeatArgs {
   double* partials;
   unsigned* tickets;
   int64_t nj, ni;
+  int64_t jb, je;  // output rows [jb, je) of the buffer (single GPU: [1, nj-1))
   int64_t ntiles;  // CTAs in the grid
 };
 
@@ -59,8 +62,8 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t c0 = ((int64_t)blockIdx.x * NW + warp) * STRIP;  // first column of my strip
   const int64_t col = c0 + (int64_t)lane * VEC;                   // my first column
-  const int64_t j0 = 1 + (int64_t)blockIdx.y * kHeatRows;
-  const int64_t j1 = min(j0 + kHeatRows, a.nj - 1);
+  const int64_t j0 = a.jb + (int64_t)blockIdx.y * kHeatRows;
+  const int64_t j1 = min(j0 + kHeatRows, a.je);
   const int64_t ni = a.ni;
   double err = 0.0;  // |d| >= 0, and the residual's initial value is 0 (C14)
 
@@ -168,8 +171,8 @@ __global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
   const int tid = threadIdx.x;
   const int64_t ni = a.ni;
   const int64_t c0 = (int64_t)blockIdx.x * kTileCols;
-  const int64_t j0 = 1 + (int64_t)blockIdx.y * kHeatRows;
-  const int64_t j1 = min(j0 + kHeatRows, a.nj - 1);  // output rows [j0, j1)
+  const int64_t j0 = a.jb + (int64_t)blockIdx.y * kHeatRows;
+  const int64_t j1 = min(j0 + kHeatRows, a.je);  // output rows [j0, j1)
   const int64_t nrows = j1 - j0 + 2;                 // loaded rows j0-1 .. j1
   // window of every row: columns [ws, we) placed at slot offset ws - (c0 - 2)
   const int64_t ws = max(c0 - 2, (int64_t)0), we = min(c0 + kTileCols + 2, ni);
@@ -249,16 +252,18 @@ __global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
   }
 }
 
-static int heat_launch(int64_t nj, int64_t ni, const double* T1, double* T2, double* residual,
-                       cudaStream_t s) {
+// Sweep output rows [jb, je) of an nj x ni buffer (rows jb-1 and je are read).
+static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
+                       double* residual, cudaStream_t s) {
   const bool v2 = (ni % 2 == 0) && ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
   const bool bulk = v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr;
   const int strip = bulk ? kTileCols : 32 * (v2 ? 2 : 1) * (kBlock / 32);
   const int64_t gx = (ni + strip - 1) / strip;
-  const int64_t gy = nj > 2 ? (nj - 2 + kHeatRows - 1) / kHeatRows : 1;
+  const int64_t gy = je > jb ? (je - jb + kHeatRows - 1) / kHeatRows : 1;
   if (gy > 65535) return XR_ERR_INVALID;
   HeatArgs a;
   a.T1 = T1; a.T2 = T2; a.residual = residual; a.nj = nj; a.ni = ni; a.ntiles = gx * gy;
+  a.jb = jb; a.je = je;
   void* partials = nullptr;
   unsigned* tickets = nullptr;
   int st = heat_workspace(s, a.ntiles * (int64_t)sizeof(double), 1, &partials, &tickets);
@@ -274,6 +279,21 @@ static int heat_launch(int64_t nj, int64_t ni, const double* T1, double* T2, dou
   return XR_OK;
 }
 
+// Row layout of rank r's slab: local rows 0 .. n+1 hold global
+// rows r*n-1 .. (r+1)*n; rows 0 and n+1 are halos (unused at the global
+// boundary).  Output rows: the owned rows minus the global boundary rows.
+int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* je) {
+  if (n_local < 1 || nranks < 1 || rank < 0 || rank >= nranks) return XR_ERR_INVALID;
+  *jb = 1 + (rank == 0 ? 1 : 0);
+  *je = n_local + 1 - (rank == nranks - 1 ? 1 : 0);
+  return XR_OK;
+}
+
+int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
+                   double* residual, cudaStream_t s) {
+  return heat_launch(nj, ni, jb, je, T1, T2, residual, s);
+}
+
 }  // namespace xr
 
 using namespace xr;
@@ -285,7 +305,39 @@ extern "C" int xr_heat_step(int64_t nj, int64_t ni, const double* T1, double* T2
   if ((nj * ni > 0) && (!T1 || !T2)) return XR_ERR_INVALID;
   if (nj > 0 && ni > 0 && (nj > (INT64_MAX / 8) / ni)) return XR_ERR_INVALID;
   if (T1 == T2 && nj * ni > 0) return XR_ERR_INVALID;
-  return heat_launch(nj, ni, T1, T2, residual, (cudaStream_t)stream);
+  return heat_launch(nj, ni, 1, nj > 2 ? nj - 1 : 1, T1, T2, residual, (cudaStream_t)stream);
+}
+
+extern "C" int xr_heat_run_sharded_sim(int64_t n_local, int64_t ni, int64_t iters, int nranks,
+                                       double* const* T1s, double* const* T2s, double* residuals,
+                                       xr_stream_t stream) {
+  if (n_local < 1 || ni < 0 || iters < 0 || nranks < 1 || !T1s || !T2s) return XR_ERR_INVALID;
+  if (iters > 0 && !residuals) return XR_ERR_INVALID;
+  cudaStream_t s = (cudaStream_t)stream;
+  const int64_t nj = n_local + 2;
+  const size_t row = (size_t)ni * sizeof(double);
+  double* tmp = nullptr;
+  if (cudaMallocAsync(&tmp, (size_t)nranks * sizeof(double), s) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+  std::vector<double*> a(T1s, T1s + nranks), b(T2s, T2s + nranks);
+  int st = XR_OK;
+  for (int64_t it = 0; it < iters && !st; ++it) {
+    for (int r = 0; r < nranks && !st; ++r) {
+      int64_t jb, je;
+      heat_slab_rows(n_local, nranks, r, &jb, &je);
+      st = heat_launch(nj, ni, jb, je, a[r], b[r], tmp + r, s);
+    }
+    // halo exchange of the new field (the NCCL path does grouped send/recv)
+    for (int r = 0; r < nranks && !st; ++r) {
+      if (r > 0 && cudaMemcpyAsync(b[r], b[r - 1] + n_local * ni, row, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        st = XR_ERR_CUDA;
+      if (r < nranks - 1 && cudaMemcpyAsync(b[r] + (n_local + 1) * ni, b[r + 1] + ni, row, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        st = XR_ERR_CUDA;
+    }
+    if (!st && gather_f64(OP_MAX, tmp, nranks, 1, residuals + it, s) != cudaSuccess) st = XR_ERR_CUDA;
+    std::swap(a, b);
+  }
+  cudaFreeAsync(tmp, s);
+  return st;
 }
 
 extern "C" int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,

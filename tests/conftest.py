@@ -18,6 +18,8 @@ def _built():
     """Compile the (CPU-side) generator and oracle once per session."""
     import datagen
     import oracle
+    import __graft_entry__
     datagen.build()
     oracle.build()
+    __graft_entry__._native().build()  # libxreduce.so (no-op when up to date)
     yield

@@ -16,8 +16,6 @@ HEADER = os.path.join(ROOT, "include", "xreduce.h")
 
 @pytest.fixture(scope="module")
 def xr():
-    from paper_conf_ppopp_xutycc14_b200 import _build
-    _build.build()
     import paper_conf_ppopp_xutycc14_b200 as m
     return m
 

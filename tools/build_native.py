@@ -1,7 +1,9 @@
 """Build libxreduce.so in-tree (nvcc, sm_100a only).
 
-Usage: python -m paper_conf_ppopp_xutycc14_b200._build [--force] [--ptxas-v]
-The .so lands next to this file so it travels with gpurun snapshots.
+Usage: python tools/build_native.py [--force] [--ptxas-v]
+The .so lands in paper_conf_ppopp_xutycc14_b200/ so it travels with gpurun
+snapshots.  This file deliberately lives OUTSIDE the package: importing the
+package loads the .so, which must not be required to build it.
 """
 from __future__ import annotations
 
@@ -10,8 +12,8 @@ import os
 import subprocess
 import sys
 
-HERE = os.path.dirname(os.path.abspath(__file__))
-ROOT = os.path.dirname(HERE)
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HERE = os.path.join(ROOT, "paper_conf_ppopp_xutycc14_b200")
 CSRC = os.path.join(HERE, "csrc")
 OBJ = os.path.join(HERE, "build")
 SO = os.path.join(HERE, "libxreduce.so")
