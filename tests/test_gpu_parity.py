@@ -267,3 +267,32 @@ def test_sharded_sim_matches_unsharded(op, dtype):
             assert st == 0
             torch.cuda.synchronize()
             check(op, dtype, gdims, levels, out.cpu().numpy(), x, init=init)
+
+
+@pytest.mark.parametrize("G,n_local,ni", [(4, 33, 130), (2, 64, 1024), (3, 20, 67), (8, 9, 520)])
+def test_heat_sharded_sim_bitwise(G, n_local, ni):
+    """Gang-row sharded heat (halo exchange + max combine) == the whole grid, bitwise."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    nj, iters = G * n_local, 12
+    T0 = oracle.heat_init(nj, ni)
+    ref_T, ref_res = oracle.heat(nj, ni, iters, T0)
+    full = T0.reshape(nj, ni)
+    t1s, t2s = [], []
+    for r in range(G):
+        slab = np.zeros((n_local + 2, ni))
+        lo, hi = r * n_local - 1, (r + 1) * n_local + 1  # global rows of the slab incl. halos
+        src_lo, src_hi = max(lo, 0), min(hi, nj)
+        slab[src_lo - lo:src_hi - lo] = full[src_lo:src_hi]
+        t1s.append(torch.from_numpy(slab.reshape(-1)).cuda())
+        t2s.append(t1s[-1].clone())
+    res = torch.zeros(iters, dtype=torch.float64, device="cuda")
+    st = xr.xr_heat_run_sharded_sim(n_local, ni, iters, [t.data_ptr() for t in t1s],
+                                    [t.data_ptr() for t in t2s], res.data_ptr(),
+                                    torch.cuda.current_stream().cuda_stream)
+    assert st == 0
+    torch.cuda.synchronize()
+    assert res.cpu().tolist() == ref_res.tolist()
+    fin = t1s if iters % 2 == 0 else t2s
+    got = np.concatenate([f.cpu().numpy().reshape(n_local + 2, ni)[1:n_local + 1] for f in fin])
+    assert np.array_equal(got.view(np.uint64), ref_T.reshape(nj, ni).view(np.uint64))
