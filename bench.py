@@ -47,14 +47,16 @@ FALLBACK_HBM_GBS = 6650.0
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
-    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="xreduce", choices=["xreduce", "reference"])
     ap.add_argument("--workload", default="fp32-sum", choices=sorted(WORKLOADS))
     ap.add_argument("--elements", type=int, default=N_PER_GPU, help="elements per GPU")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--force-comm", action="store_true",
+                    help="use the NCCL sharded path even at world size 1 (exercises xr_comm_*)")
     return ap.parse_args()
 
 
@@ -175,7 +177,7 @@ def run_reference(args):
         return 0
     wl = args.workload
     n = args.elements
-    sample_n = min(n, 1 << 26)
+    sample_n = min(n, 1 << 24)  # bounded sample per step: the whole run stays within minutes
     x = make_input(wl, sample_n, 0, n)
     per_step = []
     for i in range(args.warmup + args.steps):
@@ -206,7 +208,12 @@ def run_gpu(args):
 
     rank, world, local = dist_env()
     torch.cuda.set_device(local)
-    if world > 1:
+    use_comm = world > 1 or args.force_comm
+    if use_comm:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29533")
+        os.environ.setdefault("RANK", str(rank))
+        os.environ.setdefault("WORLD_SIZE", str(world))
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     wl = args.workload
     op, dtype, kind, esz = WORKLOADS[wl]
@@ -220,7 +227,7 @@ def run_gpu(args):
     out = torch.zeros(1, dtype=tdt, device="cuda")
     stream = torch.cuda.current_stream()
     sh = stream.cuda_stream
-    comm = xr.Comm() if world > 1 else None
+    comm = xr.Comm() if use_comm else None
 
     def step():
         if comm is None:
@@ -239,7 +246,7 @@ def run_gpu(args):
     clocks.start()
     time.sleep(0.3)  # let the sampler attach
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    if world > 1:
+    if use_comm:
         dist.barrier()
     torch.cuda.synchronize()
     launches0 = xr.xr_launch_count()
@@ -252,13 +259,13 @@ def run_gpu(args):
         ev[i][1].record(stream)
     t_end.record(stream)
     torch.cuda.synchronize()
-    if world > 1:
+    if use_comm:
         dist.barrier()
     launches = xr.xr_launch_count() - launches0
     ck = clocks.stop()
     total_ms = t_start.elapsed_time(t_end)
     per = [a.elapsed_time(b) for a, b in ev]
-    if world > 1:
+    if use_comm:
         t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         total_ms = float(t.item())
@@ -267,6 +274,10 @@ def run_gpu(args):
 
     # kernel-only duration: at N=1 the step IS the one reduction kernel
     kern_ms = statistics.mean(per)
+    plan = xr.xr_plan_describe(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), torch.cuda.get_device_properties(0).multi_processor_count)
+    kernel_name = {"stream": "stream_kernel (cp.async.bulk smem ring, single pass)",
+                   "seg": "seg_kernel", "col": "col_kernel", "coltma": "coltma_kernel"}.get(plan["kernel"], plan["kernel"]) + \
+        f" [{plan['shape']} shape, {plan['units']} units, grid {plan['grid']}]"
     peak, peak_src = peak_hbm()
     alg_bytes = n * esz + esz  # read every input element once + write one output
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
@@ -277,7 +288,7 @@ def run_gpu(args):
     if args.e2e_steps > 0:
         out_h = np.zeros(1, dtype={"fp32": np.float32, "int64": np.int64}[dtype])
         hp = host.data_ptr()
-        if world == 1:
+        if comm is None:
             xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)  # warm staging
             torch.cuda.synchronize()
             t0 = time.perf_counter()
@@ -323,7 +334,7 @@ def run_gpu(args):
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,
-                         "kernel": "seg_kernel<W=CTA> (xr_reduce R-shape)",
+                         "kernel": kernel_name,
                          "algorithmic_bytes_per_launch": alg_bytes,
                          "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)},
             "hbm_frac_of_peak": achieved / peak,
@@ -335,7 +346,7 @@ def run_gpu(args):
         print(json.dumps(line), flush=True)
     if comm is not None:
         comm.close()
-    if world > 1:
+    if use_comm:
         dist.destroy_process_group()
     return 0
 

@@ -1,0 +1,67 @@
+"""The real NCCL path with a 1-rank communicator (one GPU is all this build can
+get): xr_comm_get_unique_id / xr_comm_init over a torch.distributed group,
+xr_reduce_sharded for every collective kind, and the sharded heat step --
+checked against the oracle.  Multi-rank exchange semantics are covered by the
+single-device simulation tests and the gloo world-2 tests."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import oracle
+from datagen import recipes
+from gpu_util import check
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def comm():
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    if not dist.is_initialized():
+        with socket.socket() as s:
+            s.bind(("127.0.0.1", 0))
+            port = s.getsockname()[1]
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ["MASTER_PORT"] = str(port)
+        dist.init_process_group("gloo", rank=0, world_size=1)
+    torch.cuda.set_device(0)
+    c = xr.Comm()
+    yield c
+    c.close()
+
+
+@pytest.mark.parametrize("op,dtype,levels", [("+", "int64", "gwv"), ("max", "fp32", "g"), ("^", "int32", "gw"),
+                                             ("&&", "fp64", "gv"), ("+", "fp32", "v"), ("*", "int32", "wv")])
+def test_reduce_sharded_one_rank(comm, op, dtype, levels):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    dims = (40, 33, 65)
+    kind = {"+": "ints", "max": "maxmin", "^": "bxor", "&&": "land", "*": "mul"}[op]
+    x = recipes.make(kind, dims, oracle.mask_of(levels), dtype, 3)
+    init = recipes.make("ints", (oracle.out_count(dims, levels), 1, 1), 1, dtype, 4)
+    out = xr.reduce_sharded(torch.from_numpy(x).cuda(), comm, op, levels, nest_local=dims, init=init)
+    torch.cuda.synchronize()
+    check(op, dtype, dims, levels, out.cpu().numpy()[:init.size], x, init=init)
+
+
+def test_heat_sharded_one_rank(comm):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    nj, ni, iters = 66, 130, 9
+    T0 = oracle.heat_init(nj, ni)
+    ref_T, ref_res = oracle.heat(nj, ni, iters, T0)
+    slab = np.zeros((nj + 2, ni))
+    slab[1:nj + 1] = T0.reshape(nj, ni)
+    t1 = torch.from_numpy(slab.reshape(-1)).cuda()
+    t2 = t1.clone()
+    res = torch.zeros(iters, dtype=torch.float64, device="cuda")
+    assert xr.xr_heat_run_sharded(nj, ni, iters, t1.data_ptr(), t2.data_ptr(), res.data_ptr(), comm,
+                                  torch.cuda.current_stream().cuda_stream) == 0
+    torch.cuda.synchronize()
+    assert res.cpu().tolist() == ref_res.tolist()
+    fin = (t1 if iters % 2 == 0 else t2).cpu().numpy().reshape(nj + 2, ni)[1:nj + 1]
+    assert np.array_equal(fin.view(np.uint64), ref_T.reshape(nj, ni).view(np.uint64))
