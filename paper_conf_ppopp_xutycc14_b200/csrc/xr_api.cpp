@@ -239,6 +239,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);
+  if (p.grid_hint > 0) info->grid = std::min(info->grid, p.grid_hint);
   info->ws_bytes = p.ws_bytes;
   info->tickets = p.tickets;
   return XR_OK;

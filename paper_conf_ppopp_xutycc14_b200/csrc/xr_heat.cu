@@ -13,6 +13,7 @@
 // last-CTA tiers of xr_ops.cuh.  Arithmetic uses __dadd_rn/__dmul_rn so no FMA
 // contraction can occur (the paper disables FMA, @35389-35893), which makes
 // the result bit-identical to the oracle.
+#include <algorithm>
 #include <cstdlib>
 #include <utility>
 #include <vector>
@@ -36,6 +37,7 @@ struct HeatArgs {
   unsigned* tickets;
   int64_t nj, ni;
   int64_t jb, je;  // output rows [jb, je) of the buffer (single GPU: [1, nj-1))
+  int64_t rows;    // output rows per CTA (bulk kernel: sized for one full wave)
   int64_t ntiles;  // CTAs in the grid
 };
 
@@ -62,8 +64,8 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int64_t c0 = ((int64_t)blockIdx.x * NW + warp) * STRIP;  // first column of my strip
   const int64_t col = c0 + (int64_t)lane * VEC;                   // my first column
-  const int64_t j0 = a.jb + (int64_t)blockIdx.y * kHeatRows;
-  const int64_t j1 = min(j0 + kHeatRows, a.je);
+  const int64_t j0 = a.jb + (int64_t)blockIdx.y * a.rows;
+  const int64_t j1 = min(j0 + a.rows, a.je);
   const int64_t ni = a.ni;
   double err = 0.0;  // |d| >= 0, and the residual's initial value is 0 (C14)
 
@@ -158,38 +160,52 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
 // folds |T2 - T1| into its private max.  Bytes in flight no longer depend on
 // registers, and every T1 byte is read from HBM once per tile (halo rows and
 // columns are ~3% extra).
-constexpr int kTileCols = 2 * kBlock;          // 512 doubles = 4 KiB per row
+constexpr int kTileCols = 2 * kConsThreads;    // 512 doubles = 4 KiB per row
 constexpr int kSlotDoubles = kTileCols + 4;    // + 2-column halo on both sides
 constexpr int kHeatSlots = 8;
 
-__global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
+__global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
   using O = Op<OP_MAX, double>;
   __shared__ __align__(128) double slots[kHeatSlots][kSlotDoubles];
   __shared__ __align__(8) uint64_t full[kHeatSlots];
+  __shared__ __align__(8) uint64_t empty[kHeatSlots];
   __shared__ double smem[32];
   __shared__ int s_last;
-  const int tid = threadIdx.x;
+  const int tid0 = threadIdx.x, warp = tid0 >> 5, lane = tid0 & 31;
   const int64_t ni = a.ni;
   const int64_t c0 = (int64_t)blockIdx.x * kTileCols;
-  const int64_t j0 = a.jb + (int64_t)blockIdx.y * kHeatRows;
-  const int64_t j1 = min(j0 + kHeatRows, a.je);  // output rows [j0, j1)
-  const int64_t nrows = j1 - j0 + 2;                 // loaded rows j0-1 .. j1
+  const int64_t j0 = a.jb + (int64_t)blockIdx.y * a.rows;
+  const int64_t j1 = min(j0 + a.rows, a.je);      // output rows [j0, j1)
+  const int64_t nrows = j1 - j0 + 2;              // loaded rows j0-1 .. j1
   // window of every row: columns [ws, we) placed at slot offset ws - (c0 - 2)
   const int64_t ws = max(c0 - 2, (int64_t)0), we = min(c0 + kTileCols + 2, ni);
   const unsigned wbytes = (unsigned)((we - ws) * 8);
   const int64_t soff = ws - (c0 - 2);
-  double err = 0.0;
 
-  if (j0 < j1) {
-    if (tid == 0) {
-      for (int k = 0; k < kHeatSlots; ++k) mbar_init(&full[k], 1);
-      fence_mbar_init();
-      for (int64_t r = 0; r < min((int64_t)kHeatSlots, nrows); ++r) {
-        mbar_expect_tx(&full[r], wbytes);
-        bulk_g2s(&slots[r][soff], a.T1 + (j0 - 1 + r) * ni + ws, wbytes, &full[r]);
+  if (tid0 == 0) {
+    for (int k = 0; k < kHeatSlots; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (warp == 0) {
+    // producer warp: row q of the tile into slot q % kHeatSlots once the
+    // consumers released the row kHeatSlots earlier
+    if (lane == 0 && j0 < j1) {
+      for (int64_t q = 0; q < nrows; ++q) {
+        const int slot = (int)(q % kHeatSlots);
+        if (q >= kHeatSlots) mbar_wait(&empty[slot], (unsigned)(((q / kHeatSlots) - 1) & 1));
+        mbar_expect_tx(&full[slot], wbytes);
+        bulk_g2s(&slots[slot][soff], a.T1 + (j0 - 1 + q) * ni + ws, wbytes, &full[slot]);
       }
     }
-    __syncthreads();
+    return;
+  }
+  const int tid = tid0 - 32, cw = warp - 1;
+  double err = 0.0;
+  if (j0 < j1) {
     mbar_wait(&full[0], 0);  // row j0-1
     mbar_wait(&full[1], 0);  // row j0
     const int64_t col = c0 + 2 * tid;  // my two columns: col, col+1
@@ -220,18 +236,12 @@ __global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
         if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
         if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
       }
-      __syncthreads();  // row r-1 is dead: refill its slot kHeatSlots rows ahead
-      if (tid == 0) {
-        const int64_t nr = r - 1 + kHeatSlots;
-        if (nr < nrows) {
-          const int slot = (int)(nr % kHeatSlots);
-          mbar_expect_tx(&full[slot], wbytes);
-          bulk_g2s(&slots[slot][soff], a.T1 + (j0 - 1 + nr) * ni + ws, wbytes, &full[slot]);
-        }
-      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[(r - 1) % kHeatSlots]);  // row r-1 is dead for this warp
     }
   }
-  err = block_reduce<OP_MAX, double, kBlock>(err, smem);
+  // a2 + a3: warp and consumer-wide max, then a4: last CTA combines all CTA partials
+  err = cons_reduce<OP_MAX, double>(err, smem, cw, lane);
   const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
   if (tid == 0) {
     a.partials[cta] = err;
@@ -239,12 +249,12 @@ __global__ void __launch_bounds__(kBlock) heat_bulk_kernel(HeatArgs a) {
     const unsigned t = atomicAdd(a.tickets, 1u);
     s_last = (t == (unsigned)(a.ntiles - 1));
   }
-  __syncthreads();
+  cons_sync();
   if (s_last) {
     __threadfence();
     double w = 0.0;
-    for (int64_t k = tid; k < a.ntiles; k += kBlock) w = O::combine(w, ld_partial(a.partials + k));
-    w = block_reduce<OP_MAX, double, kBlock>(w, smem);
+    for (int64_t k = tid; k < a.ntiles; k += kConsThreads) w = O::combine(w, ld_partial(a.partials + k));
+    w = cons_reduce<OP_MAX, double>(w, smem, cw, lane);
     if (tid == 0) {
       *a.residual = w;
       *a.tickets = 0u;
@@ -259,9 +269,13 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   const bool bulk = v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr;
   const int strip = bulk ? kTileCols : 32 * (v2 ? 2 : 1) * (kBlock / 32);
   const int64_t gx = (ni + strip - 1) / strip;
-  const int64_t gy = je > jb ? (je - jb + kHeatRows - 1) / kHeatRows : 1;
+  // 64-row tiles (2048 CTAs at 8192^2).  Sizing row blocks for one full wave
+  // of resident CTAs measured slower (0.79 vs 0.89 of peak, r01), so it is not used.
+  const int64_t rows = kHeatRows;
+  const int64_t gy = je > jb ? (je - jb + rows - 1) / rows : 1;
   if (gy > 65535) return XR_ERR_INVALID;
   HeatArgs a;
+  a.rows = rows;
   a.T1 = T1; a.T2 = T2; a.residual = residual; a.nj = nj; a.ni = ni; a.ntiles = gx * gy;
   a.jb = jb; a.je = je;
   void* partials = nullptr;
@@ -271,7 +285,7 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   a.partials = static_cast<double*>(partials);
   a.tickets = tickets;
   dim3 grid((unsigned)gx, (unsigned)gy);
-  if (bulk) heat_bulk_kernel<<<grid, kBlock, 0, s>>>(a);
+  if (bulk) heat_bulk_kernel<<<grid, kWsBlock, 0, s>>>(a);
   else if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
   else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);
   count_launch();

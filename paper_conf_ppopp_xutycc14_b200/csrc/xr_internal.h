@@ -69,6 +69,7 @@ struct Plan {
   int64_t ws_bytes = 0;
   int64_t tickets = 0;
   bool sched = false;   // CTA-wide units are claimed dynamically (2 extra counters)
+  int64_t grid_hint = 0;  // >0: launch exactly this many CTAs (equal units per CTA)
   SegArgs seg{};
   ColArgs col{};
   CUtensorMap tmap{};   // K_COLTMA: 3-D map over (K, R, B), built at launch

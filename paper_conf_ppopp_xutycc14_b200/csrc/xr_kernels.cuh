@@ -270,157 +270,159 @@ __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u)
   return g;
 }
 
-template <int OP, typename T, int BLOCK, int NS, int STAGE>
-__global__ void __launch_bounds__(BLOCK) stream_kernel(SegArgs a) {
+template <int OP, typename T, int NS, int STAGE>
+__global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
-  constexpr int PER = STAGE / (16 * BLOCK);  // 16-B vectors per thread per stage
-  constexpr int RING = 8;                    // published unit ids (producer <= 3 units ahead)
-  static_assert(PER >= 1 && STAGE % (16 * BLOCK) == 0, "stage geometry");
+  constexpr int PER = STAGE / (16 * kConsThreads);  // 16-B vectors per consumer thread per stage
+  constexpr int RING = 8;                           // published unit ids
+  static_assert(PER >= 1 && STAGE % (16 * kConsThreads) == 0, "stage geometry");
   extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE
   __shared__ __align__(8) uint64_t full[NS];
+  __shared__ __align__(8) uint64_t empty[NS];
   __shared__ long long s_units[RING];
   __shared__ Acc smem[32];
   __shared__ int s_last;
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
   const int64_t S = a.Sc;
-
-  // ---- producer state (meaningful in thread 0 only)
-  long long p_unit = 0, p_next = 0;
-  int64_t p_k = 0, p_nk = 0, p_bytes = 0, g_issue = 0;
-  const char* p_src = nullptr;
-  int p_seq = 0;
-  auto p_start = [&](long long u) {
-    p_unit = u;
-    s_units[p_seq & (RING - 1)] = u < a.units ? u : -1;
-    ++p_seq;
-    p_k = 0;
-    p_nk = 0;
-    if (u < a.units) {
-      const StreamGeom g = stream_geom<T>(a, u);
-      p_src = static_cast<const char*>(g.row) + g.head * (int64_t)sizeof(T);
-      p_bytes = g.nbody * (int64_t)sizeof(T);
-      p_nk = (p_bytes + STAGE - 1) / STAGE;
-    }
-  };
-  auto p_issue = [&]() {  // issue the next chunk of the global chunk sequence, if any
-    while (p_unit < a.units && p_k == p_nk) {
-      const long long nu = p_next;
-      p_next = (long long)atomicAdd(a.sched, 1ull);  // claimed one unit ahead
-      p_start(nu);
-    }
-    if (p_unit >= a.units) return;
-    const int slot = (int)(g_issue % NS);
-    const unsigned bytes = (unsigned)min((int64_t)STAGE, p_bytes - p_k * STAGE);
-    mbar_expect_tx(&full[slot], bytes);
-    bulk_g2s(stage_mem + slot * STAGE, p_src + p_k * STAGE, bytes, &full[slot]);
-    ++p_k;
-    ++g_issue;
-  };
+  const bool whole = (a.O == 1);
 
   if (tid == 0) {
 #pragma unroll
-    for (int k = 0; k < NS; ++k) mbar_init(&full[k], 1);
+    for (int k = 0; k < NS; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
     fence_mbar_init();
-    const long long u0 = (long long)atomicAdd(a.sched, 1ull);
-    p_next = (long long)atomicAdd(a.sched, 1ull);
-    p_start(u0);
-    for (int k = 0; k < NS; ++k) p_issue();
   }
   __syncthreads();
 
-  // One output (R shape): every unit's partial goes to partials[u] with no
-  // per-unit fence or ticket; each CTA takes ONE ticket at exit and the last
-  // CTA combines the S unit partials in unit order -- deterministic although
-  // units are claimed dynamically.  Several outputs: per-unit ticket per output.
-  const bool whole = (a.O == 1);
+  if (warp == 0) {
+    // ---------------- producer warp: claims units, publishes their ids and
+    // streams their 16-B aligned bodies into the ring NS stages ahead; it never
+    // waits for the consumers' epilogues, only for a stage to be released.
+    if (lane == 0) {
+      int64_t g = 0;
+      int seq = 0;
+      long long u = (long long)atomicAdd(a.sched, 1ull);
+      while (true) {
+        const long long nu = (long long)atomicAdd(a.sched, 1ull);  // next claim, in flight
+        const int slot0 = (int)(g % NS);
+        s_units[seq & (RING - 1)] = u < a.units ? u : -1;
+        ++seq;
+        if (u >= a.units) {  // end marker: complete the next full phase without data
+          if (g >= NS) mbar_wait(&empty[slot0], (unsigned)(((g / NS) - 1) & 1));
+          mbar_arrive(&full[slot0]);
+          break;
+        }
+        const StreamGeom geo = stream_geom<T>(a, u);
+        const char* src = static_cast<const char*>(geo.row) + geo.head * (int64_t)sizeof(T);
+        const int64_t bytes = geo.nbody * (int64_t)sizeof(T);
+        const int64_t nk = (bytes + STAGE - 1) / STAGE;
+        for (int64_t k = 0; k < nk; ++k, ++g) {
+          const int slot = (int)(g % NS);
+          if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
+          const unsigned nb = (unsigned)min((int64_t)STAGE, bytes - k * STAGE);
+          mbar_expect_tx(&full[slot], nb);
+          bulk_g2s(stage_mem + slot * STAGE, src + k * STAGE, nb, &full[slot]);
+        }
+        u = nu;
+      }
+      sched_exit(a.sched);
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  const int ct = tid - 32, cw = warp - 1;
   int seq = 0;
-  int64_t g = 0;  // consumer's global chunk index (stage = g % NS, phase parity = (g / NS) & 1)
+  int64_t g = 0;
   Acc acc[PER][VEC];
 #pragma unroll
   for (int j = 0; j < PER; ++j)
 #pragma unroll
     for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
   while (true) {
+    // the first stage of the next unit (or the end marker) publishes its id
+    mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
     const StreamGeom geo = stream_geom<T>(a, u);
     const T* row = static_cast<const T*>(geo.row);
-    if (tid < geo.head) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(row + tid)));
-    if (tid < geo.tail)
-      acc[0][VEC - 1] = O::combine(acc[0][VEC - 1], O::lift(ld_scalar(row + geo.head + geo.nbody + tid)));
+    if (ct < geo.head) acc[0][0] = O::combine(acc[0][0], O::lift(ld_scalar(row + ct)));
+    if (ct < geo.tail)
+      acc[0][VEC - 1] = O::combine(acc[0][VEC - 1], O::lift(ld_scalar(row + geo.head + geo.nbody + ct)));
     const int64_t body_bytes = geo.nbody * (int64_t)sizeof(T);
     const int64_t nk = (body_bytes + STAGE - 1) / STAGE;
     for (int64_t k = 0; k < nk; ++k, ++g) {
       const int slot = (int)(g % NS);
-      mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      if (k > 0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const int64_t bytes = min((int64_t)STAGE, body_bytes - k * STAGE);
       const unsigned char* st = stage_mem + slot * STAGE;
 #pragma unroll
       for (int j = 0; j < PER; ++j) {
-        const int off = (tid + j * BLOCK) * 16;
+        const int off = (ct + j * kConsThreads) * 16;
         if (off < bytes) {
           const U128 x = *reinterpret_cast<const U128*>(st + off);
 #pragma unroll
           for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x, q)));
         }
       }
-      __syncthreads();            // every thread is done with this stage
-      if (tid == 0) p_issue();    // refill it NS chunks ahead
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);  // this warp is done with the stage
     }
     Acc v = fold_acc<OP, T, PER, VEC>(acc);
 #pragma unroll
     for (int j = 0; j < PER; ++j)
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
-    v = block_reduce<OP, T, BLOCK>(v, smem);
+    v = cons_reduce<OP, T>(v, smem, cw, lane);
     const int64_t o = geo.o;
     if (whole) {
-      if (tid == 0) partials[u] = v;
+      if (ct == 0) partials[u] = v;
     } else if (S == 1) {
-      if (tid == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+      if (ct == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
     } else {
-      if (tid == 0) {
+      if (ct == 0) {
         partials[u] = v;
         __threadfence();
         const unsigned t = atomicAdd(&a.tickets[o], 1u);
         s_last = (t == (unsigned)(S - 1));
       }
-      __syncthreads();
+      cons_sync();
       if (s_last) {
         __threadfence();
-        Acc w = fold_partials<OP, T>(partials + o * S, S, tid, BLOCK);
-        w = block_reduce<OP, T, BLOCK>(w, smem);
-        if (tid == 0) {
+        Acc w = fold_partials<OP, T>(partials + o * S, S, ct, kConsThreads);
+        w = cons_reduce<OP, T>(w, smem, cw, lane);
+        if (ct == 0) {
           out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
           a.tickets[o] = 0u;
         }
       }
     }
-    __syncthreads();
+    cons_sync();
     ++seq;
   }
-  if (whole) {  // a4: one ticket per CTA; the last CTA combines the S unit partials
-    if (tid == 0) {
+  if (whole) {  // a4: one ticket per CTA; the last CTA folds the S unit partials in unit order
+    if (ct == 0) {
       __threadfence();
       const unsigned t = atomicAdd(&a.tickets[0], 1u);
       s_last = (t == gridDim.x - 1u);
     }
-    __syncthreads();
+    cons_sync();
     if (s_last) {
       __threadfence();
-      Acc w = fold_partials<OP, T>(partials, S, tid, BLOCK);
-      w = block_reduce<OP, T, BLOCK>(w, smem);
-      if (tid == 0) {
+      Acc w = fold_partials<OP, T>(partials, S, ct, kConsThreads);
+      w = cons_reduce<OP, T>(w, smem, cw, lane);
+      if (ct == 0) {
         out[0] = merge_init<OP, T>(w, out, 0, a.init_from_out);
         a.tickets[0] = 0u;
       }
     }
   }
-  sched_exit(a.sched);
 }
 
 // ------------------------------------------------------------- col kernel
@@ -560,79 +562,83 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
 // the worker tier folds the row phases per column in shared memory; the gang
 // tier is the per-tile ticket of col_kernel.  OOB rows/columns of a box are
 // skipped by the consumers, so the fill value never matters.
-template <int OP, typename T, int BLOCK, int NS>
-__global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
+template <int OP, typename T, int NS>
+__global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
+  constexpr int BLOCK = kConsThreads;        // consumer threads
   constexpr int VEC = 16 / sizeof(T);
   constexpr int TW = 1024 / (int)sizeof(T);  // box columns
   constexpr int BR = kStageBytes / 1024;     // box rows
   constexpr int G = TW / VEC;                // 16-B column groups per row
   constexpr int NPH = BLOCK / G;             // row phases
-  constexpr int PH2 = BLOCK / TW;            // threads per column in the tile combine
   constexpr int RING = 8;
   constexpr int AV = 16 / (int)sizeof(Acc);  // partials per 16-B load in the folds
   constexpr int NPA = BLOCK / (TW / AV);     // row phases of the folds
   constexpr int NRED = NPH > NPA ? NPH : NPA;
-  static_assert(NPH >= 1 && PH2 >= 1 && NPA >= 1 && BR % NPH == 0, "geometry");
+  static_assert(NPH >= 1 && NPA >= 1 && BR % NPH == 0, "geometry");
   extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * kStageBytes
   __shared__ __align__(8) uint64_t full[NS];
+  __shared__ __align__(8) uint64_t empty[NS];
   __shared__ long long s_units[RING];
   __shared__ __align__(16) Acc red[NRED][TW];
   __shared__ int s_last;
-  const int tid = threadIdx.x, grp = tid % G, ph = tid / G;
+  const int tid0 = threadIdx.x, warp = tid0 >> 5, lane = tid0 & 31;
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
   const int64_t per_b = a.tiles * a.S;
 
-  // ---- producer (thread 0)
-  long long p_unit = 0, p_next = 0;
-  int64_t p_k = 0, p_nk = 0, g_issue = 0, p_b = 0, p_tile = 0, p_r0 = 0;
-  int p_seq = 0;
-  auto p_start = [&](long long u) {
-    p_unit = u;
-    s_units[p_seq & (RING - 1)] = u < a.units ? u : -1;
-    ++p_seq;
-    p_k = 0;
-    p_nk = 0;
-    if (u < a.units) {
-      p_b = u / per_b;
-      const int64_t rem = u - p_b * per_b;
-      p_tile = rem / a.S;
-      const int64_t s = rem - p_tile * a.S;
-      p_r0 = split_lo(a.R, a.S, s);
-      p_nk = (split_lo(a.R, a.S, s + 1) - p_r0 + BR - 1) / BR;
-    }
-  };
-  auto p_issue = [&]() {
-    while (p_unit < a.units && p_k == p_nk) {
-      const long long nu = p_next;
-      p_next = (long long)atomicAdd(a.sched, 1ull);
-      p_start(nu);
-    }
-    if (p_unit >= a.units) return;
-    const int slot = (int)(g_issue % NS);
-    mbar_expect_tx(&full[slot], (unsigned)kStageBytes);
-    tma_load_3d(stage_mem + slot * kStageBytes, &tmap, (int)(p_tile * TW), (int)(p_r0 + p_k * BR), (int)p_b,
-                &full[slot]);
-    ++p_k;
-    ++g_issue;
-  };
-  if (tid == 0) {
+  if (tid0 == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
 #pragma unroll
-    for (int k = 0; k < NS; ++k) mbar_init(&full[k], 1);
+    for (int k = 0; k < NS; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
     fence_mbar_init();
-    const long long u0 = (long long)atomicAdd(a.sched, 1ull);
-    p_next = (long long)atomicAdd(a.sched, 1ull);
-    p_start(u0);
-    for (int k = 0; k < NS; ++k) p_issue();
   }
   __syncthreads();
 
+  if (warp == 0) {
+    // ---------------- producer warp
+    if (lane == 0) {
+      int64_t g = 0;
+      int seq = 0;
+      long long u = (long long)atomicAdd(a.sched, 1ull);
+      while (true) {
+        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const int slot0 = (int)(g % NS);
+        s_units[seq & (RING - 1)] = u < a.units ? u : -1;
+        ++seq;
+        if (u >= a.units) {
+          if (g >= NS) mbar_wait(&empty[slot0], (unsigned)(((g / NS) - 1) & 1));
+          mbar_arrive(&full[slot0]);
+          break;
+        }
+        const int64_t b = u / per_b, rem = u - b * per_b;
+        const int64_t tile = rem / a.S, s = rem - tile * a.S;
+        const int64_t r0 = split_lo(a.R, a.S, s), r1 = split_lo(a.R, a.S, s + 1);
+        const int64_t nk = (r1 - r0 + BR - 1) / BR;
+        for (int64_t k = 0; k < nk; ++k, ++g) {
+          const int slot = (int)(g % NS);
+          if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
+          mbar_expect_tx(&full[slot], (unsigned)kStageBytes);
+          tma_load_3d(stage_mem + slot * kStageBytes, &tmap, (int)(tile * TW), (int)(r0 + k * BR), (int)b,
+                      &full[slot]);
+        }
+        u = nu;
+      }
+      sched_exit(a.sched);
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  const int tid = tid0 - 32, grp = tid % G, ph = tid / G;
   int seq = 0;
   int64_t g = 0;
   while (true) {
+    mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
     const int64_t b = u / per_b, rem = u - b * per_b;
@@ -647,7 +653,7 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
       for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
     for (int64_t k = 0; k < nk; ++k, ++g) {
       const int slot = (int)(g % NS);
-      mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      if (k > 0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const unsigned char* st = stage_mem + slot * kStageBytes;
       const int64_t rbase = r0 + k * BR;
 #pragma unroll
@@ -659,13 +665,13 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
           for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
         }
       }
-      __syncthreads();
-      if (tid == 0) p_issue();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);
     }
     // a3: fold the row phases per column
 #pragma unroll
     for (int q = 0; q < VEC; ++q) red[ph][grp * VEC + q] = O::combine(acc[0][q], acc[1][q]);
-    __syncthreads();
+    cons_sync();
     const int64_t oc = tile * TW + tid;  // output column of thread tid (< TW)
     Acc v = O::identity();
     if (tid < TW) {
@@ -676,8 +682,7 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
       if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(v, out, b * a.K + oc, a.init_from_out);
     } else {
       // a4, two levels: unit partial -> group of kGroupFold (its last CTA folds
-      // the group in unit order) -> tile (the last group folds the G2 group
-      // partials).  Keeps every fold short although S can be ~1000.
+      // the group in unit order) -> tile (the last group folds the G2 group partials)
       const int64_t tid_tile = b * a.tiles + tile;
       Acc* P1 = partials + tid_tile * a.S * TW;                                  // [S][TW]
       Acc* P2 = partials + a.B * a.tiles * a.S * TW + tid_tile * a.G2 * TW;      // [G2][TW]
@@ -709,7 +714,7 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
         }
 #pragma unroll
         for (int q = 0; q < AV; ++q) red[q2][cg * AV + q] = w[q];
-        __syncthreads();
+        cons_sync();
         Acc z = O::identity();
         if (tid < TW) {
 #pragma unroll
@@ -718,13 +723,13 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
         return z;
       };
       if (tid < TW) P1[s * TW + tid] = v;
-      __syncthreads();  // partial stores happen-before thread 0's (cumulative) fence
+      cons_sync();  // partial stores happen-before thread 0's (cumulative) fence
       if (tid == 0) {
         __threadfence();
         const unsigned tk = atomicAdd(&gt[grp_i], 1u);
         s_last = (tk == (unsigned)(gsz - 1));
       }
-      __syncthreads();
+      cons_sync();
       if (s_last) {
         __threadfence();
         const Acc w = fold_rows(P1 + g0 * TW, gsz);
@@ -733,13 +738,13 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
           if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(w, out, b * a.K + oc, a.init_from_out);
         } else {
           if (tid < TW) P2[grp_i * TW + tid] = w;
-          __syncthreads();
+          cons_sync();
           if (tid == 0) {
             __threadfence();
             const unsigned tk = atomicAdd(tt, 1u);
             s_last = (tk == (unsigned)(a.G2 - 1));
           }
-          __syncthreads();
+          cons_sync();
           if (s_last) {
             __threadfence();
             const Acc z = fold_rows(P2, a.G2);
@@ -749,10 +754,9 @@ __global__ void __launch_bounds__(BLOCK) coltma_kernel(const __grid_constant__ C
         }
       }
     }
-    __syncthreads();
+    cons_sync();
     ++seq;
   }
-  sched_exit(a.sched);
 }
 
 // ------------------------------------------------------------- elementwise
@@ -824,27 +828,29 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       break;
     }
     case K_STREAM: {
-      auto kern = stream_kernel<OP, T, kBlock, kStages, kStageBytes>;
+      auto kern = stream_kernel<OP, T, kStages, kStageBytes>;
       constexpr int dyn = kStages * kStageBytes;
       static int occ = [&] {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
         return n;
       }();
-      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, dyn, s>>>(p.seg);
+      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_COLTMA: {
-      auto kern = coltma_kernel<OP, T, kBlock, kStages>;
+      auto kern = coltma_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
       static int occ = [&] {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
         return n;
       }();
-      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, dyn, s>>>(p.tmap, p.col);
+      int64_t grid = grid_for(p.units, num_sms, occ);
+      if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
+      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.tmap, p.col);
       break;
     }
     case K_COL: {

@@ -272,3 +272,35 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
       : "memory");
 }
 }  // namespace xr
+
+namespace xr {
+// ------------------------------------------------------------ warp specialisation
+// Producer warp + kConsWarps consumer warps: the consumers synchronise among
+// themselves with named barrier 1 (never with the producer), and release a
+// stage by one arrival per consumer warp on its "empty" mbarrier.
+constexpr int kConsWarps = 8;
+constexpr int kConsThreads = 32 * kConsWarps;
+constexpr int kWsBlock = kConsThreads + 32;  // + the producer warp
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
+}
+__device__ __forceinline__ void cons_sync() {
+  asm volatile("bar.sync 1, %0;" ::"n"(kConsThreads) : "memory");
+}
+// Consumer-wide combine (a2 + a3); result valid in consumer warp 0.  The
+// caller must cons_sync() before reusing smem.
+template <int OP, typename T>
+__device__ __forceinline__ typename Op<OP, T>::Acc cons_reduce(typename Op<OP, T>::Acc v,
+                                                               typename Op<OP, T>::Acc* smem, int cw,
+                                                               int lane) {
+  v = group_reduce<OP, T, 32>(v);
+  if (lane == 0) smem[cw] = v;
+  cons_sync();
+  if (cw == 0) {
+    v = lane < kConsWarps ? smem[lane] : Op<OP, T>::identity();
+    v = group_reduce<OP, T, 32>(v);
+  }
+  return v;
+}
+}  // namespace xr

@@ -105,19 +105,33 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
         B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {
       const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
       const int64_t tiles = cdiv(K, TWt);
-      // ~8 units per resident CTA (3 per SM): a CTA streams ~16.5 GB/s, so the
-      // tail is about one unit (r01i: 4 per CTA left SMs idle 25% of the time),
-      // while each unit still amortises its epilogue (r01j: 16 per CTA too many)
-      const int64_t target = 8 * (int64_t)std::max(num_sms, 1) * 3;
-      int64_t S = cdiv(target, B * tiles);
-      S = std::min<int64_t>(S, std::max<int64_t>(1, R / (kStages * BR)));  // >= kStages boxes per unit
-
+      // Balance (measured r01 sweeps): the producer warp keeps every CTA's ring
+      // full, so few long units per CTA are best, but the unit count must be an
+      // exact multiple of the CTAs launched (896 units on 444 CTAs left 8
+      // stragglers for a third round).  k units per CTA, grid = units / k.
+      const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;  // resident CTAs (64 KiB ring each)
+      const int64_t base = B * tiles;
+      const char* upc = std::getenv("XR_COLTMA_UNITS_PER_CTA");  // tuning override
+      // measured (r01 sweeps): 2 units per CTA is best with few column tiles
+      // (512^3 G/W/GW: 0.95/0.95/0.97 at 1 GiB); with many tiles (cfg3: 128)
+      // ~512 KiB units (up to 16 per CTA) win (1.04 vs 1.02)
+      const int64_t k_auto = base >= 64
+          ? std::min<int64_t>(16, std::max<int64_t>(2, (B * R * K * size) / (cap << 19))) : 2;
+      const int64_t k = upc ? std::max(1, std::atoi(upc)) : k_auto;
+      int64_t S;
+      if (base >= k * cap) {
+        S = 1;
+      } else {
+        S = std::max<int64_t>(1, (k * cap) / base);
+        S = std::min<int64_t>(S, std::max<int64_t>(1, R / (kStages * BR)));  // >= kStages boxes per unit
+      }
       if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * 8));
       S = std::max<int64_t>(1, std::min<int64_t>(S, R));
       p->kernel = K_COLTMA;
       p->vec = vec;
       p->splits = S;
       p->units = B * tiles * S;
+      p->grid_hint = std::min<int64_t>(cap, cdiv(p->units, std::max<int64_t>(k, cdiv(p->units, cap))));
       p->group = kBlock;
       p->sched = true;
       // two-level gang tier: groups of kGroupFold unit partials, then the groups
