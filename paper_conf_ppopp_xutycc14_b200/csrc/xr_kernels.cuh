@@ -26,6 +26,14 @@ __device__ __forceinline__ int64_t split_lo_vec(int64_t n, int64_t parts, int64_
   return (split_lo(n, parts, i) / v) * v;
 }
 
+// Rows [r0, r1) of split s when R rows are split in S parts at whole boxes of
+// BR rows (no TMA box straddles two units, so no row is fetched twice).
+__device__ __forceinline__ void box_rows(int64_t R, int64_t S, int64_t s, int BR, int64_t* r0, int64_t* r1) {
+  const int64_t nb = (R + BR - 1) / BR;
+  *r0 = min(split_lo(nb, S, s) * BR, R);
+  *r1 = min(split_lo(nb, S, s + 1) * BR, R);
+}
+
 // ------------------------------------------------------------- a1 (rows)
 // Fold row[0..n) into the lane's private accumulators: a scalar head up to the
 // first 16-B boundary, 16-B vectors strided by the group width W with U loads
@@ -617,7 +625,8 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
         }
         const int64_t b = u / per_b, rem = u - b * per_b;
         const int64_t tile = rem / a.S, s = rem - tile * a.S;
-        const int64_t r0 = split_lo(a.R, a.S, s), r1 = split_lo(a.R, a.S, s + 1);
+        int64_t r0, r1;
+        box_rows(a.R, a.S, s, BR, &r0, &r1);
         const int64_t nk = (r1 - r0 + BR - 1) / BR;
         for (int64_t k = 0; k < nk; ++k, ++g) {
           const int slot = (int)(g % NS);
@@ -643,7 +652,8 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
     if (u < 0) break;
     const int64_t b = u / per_b, rem = u - b * per_b;
     const int64_t tile = rem / a.S, s = rem - tile * a.S;
-    const int64_t r0 = split_lo(a.R, a.S, s), r1 = split_lo(a.R, a.S, s + 1);
+    int64_t r0, r1;
+    box_rows(a.R, a.S, s, BR, &r0, &r1);
     const int64_t nk = (r1 - r0 + BR - 1) / BR;
     const bool col_ok = tile * TW + (int64_t)grp * VEC < a.K;  // K % VEC == 0: whole vectors
     Acc acc[2][VEC];
