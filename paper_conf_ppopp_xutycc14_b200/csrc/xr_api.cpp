@@ -235,7 +235,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   info->units = p.units;
   info->block = p.block;
   int64_t ctas = p.units;
-  if (p.kernel == K_STREAM || p.kernel == K_COLTMA) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
+  if (p.kernel == K_STREAM || p.kernel == K_COLTMA || p.kernel == K_ROWS) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);

@@ -433,6 +433,127 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
   }
 }
 
+// ------------------------------------------------------------- rows kernel
+// KR with short rows (row_bytes a power of two in [512 B, 2 KiB], 16-B
+// aligned): consecutive rows are one contiguous range, so a unit is a block of
+// whole 16 KiB stages (RPS = 16 KiB / row_bytes >= 8 rows each), streamed by
+// the producer warp with cp.async.bulk.  Consumer warp w owns rows
+// w*RPW .. w*RPW+RPW-1 of every stage (RPW = RPS / 8): its lanes fold the
+// row's 16-B vectors, one warp reduction (a2) per row, lane 0 writes the
+// output (merging init).  No shared-memory combine and no barrier per stage
+// (a first version with per-stage slot folds was consumer bound, r01), and
+// rows never span CTAs, so there is no gang tier.
+template <int OP, typename T, int NS>
+__global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int STAGE = kStageBytes;
+  constexpr int RING = 8;
+  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE
+  __shared__ __align__(8) uint64_t full[NS];
+  __shared__ __align__(8) uint64_t empty[NS];
+  __shared__ long long s_units[RING];
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  T* out = static_cast<T*>(a.out);
+  const int64_t row_bytes = a.L * (int64_t)sizeof(T);
+  const int rshift = __ffsll(row_bytes) - 1;                 // row_bytes is a power of two
+  const int rps = (int)(STAGE >> rshift);                     // rows per full stage
+  const int64_t nst = (a.O + rps - 1) / rps;                  // stages overall
+  const int64_t S = a.Sc;                                     // units (blocks of stages)
+
+  if (tid == 0) {
+#pragma unroll
+    for (int k = 0; k < NS; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  if (warp == 0) {  // ---------------- producer warp
+    if (lane == 0) {
+      int64_t g = 0;
+      int seq = 0;
+      long long u = (long long)atomicAdd(a.sched, 1ull);
+      while (true) {
+        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const int slot0 = (int)(g % NS);
+        s_units[seq & (RING - 1)] = u < S ? u : -1;
+        ++seq;
+        if (u >= S) {
+          if (g >= NS) mbar_wait(&empty[slot0], (unsigned)(((g / NS) - 1) & 1));
+          mbar_arrive(&full[slot0]);
+          break;
+        }
+        const int64_t st0 = split_lo(nst, S, u), st1 = split_lo(nst, S, u + 1);
+        for (int64_t st = st0; st < st1; ++st, ++g) {
+          const int slot = (int)(g % NS);
+          if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
+          const int64_t row0 = st * rps;
+          const unsigned nb = (unsigned)(min((int64_t)rps, a.O - row0) << rshift);
+          mbar_expect_tx(&full[slot], nb);
+          bulk_g2s(stage_mem + slot * STAGE, static_cast<const char*>(a.in) + (row0 << rshift), nb, &full[slot]);
+        }
+        u = nu;
+      }
+      sched_exit(a.sched);
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  const int cw = warp - 1;
+  int seq = 0;
+  int64_t g = 0;
+  while (true) {
+    mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
+    const long long u = s_units[seq & (RING - 1)];
+    if (u < 0) break;
+    const int64_t st0 = split_lo(nst, S, u), st1 = split_lo(nst, S, u + 1);
+    for (int64_t st = st0; st < st1; ++st, ++g) {
+      const int slot = (int)(g % NS);
+      if (st > st0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      const int64_t row0 = st * rps;
+      const int nrows = (int)min((int64_t)rps, a.O - row0);
+      const unsigned char* sm = stage_mem + slot * STAGE;
+      const int rpw = rps / kConsWarps;                 // rows per warp (1, 2 or 4)
+      const int vpl = (int)(row_bytes >> 9);            // 16-B vectors per lane per row (1..4)
+      Acc v[4];
+#pragma unroll
+      for (int rr = 0; rr < 4; ++rr) {
+        v[rr] = O::identity();
+        const int r = cw * rpw + rr;
+        if (rr < rpw && r < nrows) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            if (k < vpl) {
+              const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + (k * 32 + lane) * 16);
+#pragma unroll
+              for (int q = 0; q < VEC; ++q) v[rr] = O::combine(v[rr], O::lift(unpack<T>(x, q)));
+            }
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);  // the stage is consumed into registers
+#pragma unroll
+      for (int rr = 0; rr < 4; ++rr) {
+        if (rr < rpw) {  // warp-uniform
+          const Acc w = group_reduce<OP, T, 32>(v[rr]);
+          const int r = cw * rpw + rr;
+          if (lane == 0 && r < nrows) {
+            const int64_t o = row0 + r;
+            out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+          }
+        }
+      }
+    }
+    ++seq;
+  }
+}
+
 // ------------------------------------------------------------- col kernel
 // Lanes own VEC contiguous kept columns (a 32*VEC-column tile per warp row);
 // the CTA's warps stride over the reduced rows of a row chunk; the worker tier
@@ -847,6 +968,20 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
         return n;
       }();
       kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsBlock, dyn, s>>>(p.seg);
+      break;
+    }
+    case K_ROWS: {
+      auto kern = rows_kernel<OP, T, kStages>;
+      constexpr int dyn = kStages * kStageBytes;
+      static int occ = [&] {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        return n;
+      }();
+      int64_t grid = grid_for(p.units, num_sms, occ);
+      if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
+      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_COLTMA: {

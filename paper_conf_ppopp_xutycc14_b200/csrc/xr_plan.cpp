@@ -178,6 +178,27 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   else { O = run_n[1]; C = run_n[0]; L = run_n[2]; rowStride = O * L; oStride = L; p->shape = XR_SHAPE_RKR; }
 
   const int64_t row_bytes = L * size;
+  // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
+  // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
+  if (nr == 2 && row_bytes >= 512 && row_bytes <= 2048 && (row_bytes & (row_bytes - 1)) == 0 &&
+      in_addr % 16 == 0 && std::getenv("XR_NO_BULK") == nullptr) {
+    const int64_t rps = kStageBytes / row_bytes;
+    const int64_t nst = cdiv(O, rps);
+    const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;
+    const int64_t k = 2;  // equal units per CTA (see the column kernel)
+    const int64_t units = std::max<int64_t>(1, std::min<int64_t>(nst / kStages, k * cap));
+    p->kernel = K_ROWS;
+    p->group = 32;
+    p->vec = vec;
+    p->splits = 1;
+    p->units = units;
+    p->sched = true;
+    p->grid_hint = std::min<int64_t>(cap, cdiv(units, k));
+    SegArgs& s = p->seg;
+    s.O = O; s.C = 1; s.L = L; s.rowStride = 0; s.oStride = L;
+    s.Sr = 1; s.Sc = units; s.units = units;
+    return;
+  }
   int W = row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };

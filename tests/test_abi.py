@@ -106,7 +106,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     shape, cd = SHAPE_TABLE[levels]
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
-    assert p["kernel"] in (("col", "coltma") if shape in ("RK", "KRK") else ("seg", "stream"))
+    assert p["kernel"] in (("col", "coltma") if shape in ("RK", "KRK") else ("seg", "stream", "rows"))
 
 
 def test_plan_canonical_cfg2_cfg3_cfg5(xr):
@@ -147,7 +147,9 @@ def test_plan_fp32_chain_cap(xr, case):
     """fp32 '+' keeps every accumulator's sequential chain <= 4096 (C9)."""
     _, dims, lv = case
     p = xr.xr_plan_describe("+", "fp32", dims, lv, 256)
-    if p["kernel"] in ("seg", "stream"):
+    if p["kernel"] == "rows":
+        per_acc = p["cdims"][1] / (32 * p["vec"])  # one row per warp-wide fold, VEC chains per lane
+    elif p["kernel"] in ("seg", "stream"):
         c = p["cdims"]
         work = {"R": c[0], "KR": c[1], "RKR": c[0] * c[2]}[p["shape"]]
         per_acc = work / p["splits"] / (p["group"] * p["vec"] * 4)

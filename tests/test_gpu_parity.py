@@ -296,3 +296,20 @@ def test_heat_sharded_sim_bitwise(G, n_local, ni):
     fin = t1s if iters % 2 == 0 else t2s
     got = np.concatenate([f.cpu().numpy().reshape(n_local + 2, ni)[1:n_local + 1] for f in fin])
     assert np.array_equal(got.view(np.uint64), ref_T.reshape(nj, ni).view(np.uint64))
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [512, 1024, 2048, 4096, 8192, 16384])
+def test_rows_kernel_short_rows(dtype, row_bytes):
+    """KR with power-of-two rows of 512 B .. 16 KiB (the bulk-streamed rows
+    kernel), ragged row counts (not a multiple of rows per stage), with init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for O, op in [(7, "+"), (1003, "max"), (4096 + 5, "&&")]:
+        dims = (O, 1, L)
+        plan = xr.xr_plan_describe(op, dtype, dims, "v", 256)
+        x = recipes.make(KIND[op], dims, 4, dtype, O)
+        init = recipes.make("ints", (O, 1, 1), 1, dtype, 2)
+        check(op, dtype, dims, "v", gpu_reduce(op, dtype, dims, "v", x, init=init), x, init=init)
+        if O >= 1003 and row_bytes <= 2048:
+            assert plan["kernel"] == "rows"
