@@ -7,6 +7,8 @@ cross-checked against the library header by tests/test_abi.py.
 
 Parity status per function:
   reduce      pinned: P1-P11, P13, P16 (tests/test_oracle_pins.py)
+  transform_reduce  pinned: P15 (lattice count by integer brute force, statistical pi),
+              dot closed forms (tests/test_oracle_pins_n1.py)
   heat        pinned: P14 (hand-derived residuals in tests/golden/, invariants)
   (the paper prints no result value for any case: its Table 2 / Fig 11-12 are
   timings only, so paper *timings* are "parity unpinned" -- context only)
@@ -55,6 +57,7 @@ def lib():
         vp = ctypes.c_void_p
         L.xro_out_count.argtypes = [i64p, ctypes.c_uint, i64p]
         L.xro_reduce.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_uint, vp, vp, vp]
+        L.xro_transform_reduce.argtypes = [ctypes.c_int, ctypes.c_int, i64p, ctypes.c_uint, vp, vp, vp, vp]
         L.xro_heat_init.argtypes = [ctypes.c_int64, ctypes.c_int64, vp]
         L.xro_heat.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, vp, vp, vp]
         _lib = L
@@ -110,6 +113,32 @@ def reduce(op: str, dtype: str, dims, levels, x: np.ndarray, init: np.ndarray | 
     st = lib().xro_reduce(OPS[op], DTYPES[dtype], _dims(dims), mask,
                           x.ctypes.data if x.size else None,
                           out.ctypes.data if n else None, S.ctypes.data)
+    if st:
+        raise OracleError(st)
+    return (out, S[:n]) if want_abs else out
+
+
+XFORMS = {"disk": 1, "dot": 2}
+
+
+def transform_reduce(xform: str, dtype: str, dims, levels, x: np.ndarray, y: np.ndarray,
+                     init: np.ndarray | None = None, want_abs: bool = False):
+    """N1 transform-reduce (see xro.h): 'disk' -> int64 counts, 'dot' -> dtype sums."""
+    mask = mask_of(levels)
+    dt = np.dtype(NP_DTYPES[dtype])
+    x = np.ascontiguousarray(x, dtype=dt).reshape(-1)
+    y = np.ascontiguousarray(y, dtype=dt).reshape(-1)
+    n = out_count(dims, mask)
+    odt = np.int64 if xform == "disk" else dt
+    if init is not None:
+        out = np.ascontiguousarray(np.asarray(init, dtype=odt).reshape(-1)).copy()
+        mask |= INIT_FROM_OUT
+    else:
+        out = np.zeros(n, odt)
+    S = np.zeros(max(n, 1), np.float64)
+    st = lib().xro_transform_reduce(XFORMS[xform], DTYPES[dtype], _dims(dims), mask,
+                                    x.ctypes.data if x.size else None, y.ctypes.data if y.size else None,
+                                    out.ctypes.data if n else None, S.ctypes.data)
     if st:
         raise OracleError(st)
     return (out, S[:n]) if want_abs else out

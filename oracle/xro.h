@@ -53,6 +53,18 @@ int xro_out_count(const int64_t dims[3], unsigned mask, int64_t* count);
 int xro_reduce(int op, int dtype, const int64_t dims[3], unsigned mask,
                const void* in, void* out, double* abs_sum);
 
+/* Transform-reduce, two inputs x, y of the same nest:
+ *  XRO_XF_DISK: Monte Carlo pi, Fig 13(c) (PAPER.md @43561-44280, 4. @42177-
+ *    47503): out[o] (int64) = init + #{ r : x*x + y*y < 1 }, the products and
+ *    the sum rounded in dtype (fp32 / fp64), no FMA (the paper disables FMA,
+ *    @35389) -- the predicate is decided in the same precision on both sides.
+ *  XRO_XF_DOT: inner product, Fig 13(b) (@41386-42177): out[o] (dtype) =
+ *    init + sum_r x*y, ints wrapping, fp in wide precision (C9 bound).
+ * abs_sum (nullable, DOT only): |init| + sum |x*y| per output. */
+enum { XRO_XF_DISK = 1, XRO_XF_DOT = 2 };
+int xro_transform_reduce(int xform, int dtype, const int64_t dims[3], unsigned mask,
+                         const void* x, const void* y, void* out, double* abs_sum);
+
 /* Heat equation (config 4, reading C14): T[j][i], nj x ni, row-major fp64. */
 int xro_heat_init(int64_t nj, int64_t ni, double* T);
 /* iters Jacobi sweeps starting from T1 (T2 must carry the same boundary);
