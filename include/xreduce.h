@@ -125,6 +125,21 @@ const char* xr_strerror(int status);
 int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                    const void* in_host, void* out_host, xr_stream_t stream);
 
+/* Transform-reduce (the loop body before the reduction), two
+ * inputs of the same nest (DEVICE, dtype-aligned, caller-owned):
+ *   XR_XF_DISK  Monte Carlo pi, Fig 13(c) (@43561-44280, section 4
+ *               @42177-47503): out[o] = init + #{ x*x + y*y < 1 } as int64,
+ *               every operation rounded in dtype (fp32/fp64 only; other dtypes
+ *               XR_ERR_UNSUPPORTED), no FMA (@35389).  out is int64.
+ *   XR_XF_DOT   inner product, Fig 13(b) (@41386-42177): out[o] = init +
+ *               sum x*y in dtype (ints wrap, C6; fp within the C9 bound).
+ * level_mask as xr_reduce.  Canonical shapes R, KR, RKR and K are supported;
+ * column shapes (RK, KRK: the reduced levels are all outside a kept
+ * contiguous level) return XR_ERR_UNSUPPORTED.  One launch, single pass. */
+typedef enum { XR_XF_DISK = 1, XR_XF_DOT = 2 } xr_xform;
+int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+                        const void* x, const void* y, void* out, xr_stream_t stream);
+
 /* ------------------------------------------------------------ planning ---- */
 
 /* Canonical shapes after dropping extent-1 levels and merging adjacent levels

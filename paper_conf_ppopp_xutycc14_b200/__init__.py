@@ -91,6 +91,7 @@ _SIGS = {
     "xr_comm_destroy": (_c, [_vp]),
     "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
+    "xr_transform_reduce": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_heat_step_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded_sim": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _c, ctypes.POINTER(_vp),
@@ -191,6 +192,16 @@ def xr_reduce_sharded_sim(op, dtype, local_dims, level_mask, shard_ptrs, out_ptr
     arr = (_vp * len(shard_ptrs))(*shard_ptrs)
     return _lib.xr_reduce_sharded_sim(_op(op), _dt(dtype), _dims(local_dims), mask_of(level_mask),
                                       arr, len(shard_ptrs), out_ptr, stream or None)
+
+
+XFORMS = {"disk": 1, "dot": 2}
+
+
+def xr_transform_reduce(xform, dtype, nest_dims, level_mask, x_ptr: int, y_ptr: int, out_ptr: int,
+                        stream: int = 0) -> int:
+    return _lib.xr_transform_reduce(XFORMS[xform] if isinstance(xform, str) else int(xform), _dt(dtype),
+                                    _dims(nest_dims), mask_of(level_mask), x_ptr or None, y_ptr or None,
+                                    out_ptr or None, stream or None)
 
 
 def xr_heat_run_sharded_sim(n_local, ni, iters, t1_ptrs, t2_ptrs, residuals_ptr, stream: int = 0) -> int:

@@ -408,6 +408,18 @@ int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask,
 cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s) {
   return gather_dtype(op, dtype, g, nranks, n, out, s);
 }
+// used by xr_xform.cu: the same per-(device, stream) workspace
+int xform_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  std::lock_guard<std::mutex> lock(g_mu);
+  Workspace& w = g_ws[{dev, (uintptr_t)s}];
+  int st = ensure_ws(w, pbytes, ntick, s);
+  if (st) return st;
+  *partials = w.partials;
+  *tickets = w.tickets;
+  return XR_OK;
+}
 // used by xr_heat.cu: the same per-(device, stream) workspace
 int heat_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets) {
   int dev = 0;

@@ -78,8 +78,10 @@ struct Plan {
 
 // Pure host: validation happens before (api.cpp).  in_addr only matters for
 // its alignment (16-B vector path of the column kernel).
+// seg_only: plan for the register seg decomposition only, with CTA-wide
+// groups (no stream / rows / TMA kernels) -- used by the transform-reduce.
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p);
+               int num_sms, Plan* p, bool seg_only = false);
 
 int dtype_size(int dtype);
 int acc_size(int op, int dtype);

@@ -35,7 +35,7 @@ int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
 }
 
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p) {
+               int num_sms, Plan* p, bool seg_only) {
   *p = Plan();
   const int size = dtype_size(dtype);
   const int vec = 16 / size;
@@ -100,6 +100,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     else { B = run_n[0]; R = run_n[1]; K = run_n[2]; p->shape = XR_SHAPE_KRK; }
     const bool aligned = ((K * size) % 16 == 0) && (in_addr % 16 == 0);
     const int cv = aligned ? vec : 1;
+    if (seg_only) {
+      p->kernel = K_COL;
+      return;
+    }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
     if (aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {
@@ -180,7 +184,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   const int64_t row_bytes = L * size;
   // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
   // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
-  if (nr == 2 && row_bytes >= 512 && row_bytes <= 2048 && (row_bytes & (row_bytes - 1)) == 0 &&
+  if (!seg_only && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 && (row_bytes & (row_bytes - 1)) == 0 &&
       in_addr % 16 == 0 && std::getenv("XR_NO_BULK") == nullptr) {
     const int64_t rps = kStageBytes / row_bytes;
     const int64_t nst = cdiv(O, rps);
@@ -199,7 +203,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     s.Sr = 1; s.Sc = units; s.units = units;
     return;
   }
-  int W = row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
+  int W = seg_only ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
   const int64_t work = C * L;  // elements per output
@@ -213,7 +217,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // long contiguous rows (R, KR): the bulk-copy stream kernel; every unit must
   // cover at least kStages stages so the producer stays <= 3 units ahead
   const int64_t stage_elems = kStageBytes / size;
-  const bool stream = C == 1 && row_bytes >= (int64_t)kStages * kStageBytes && std::getenv("XR_NO_BULK") == nullptr;
+  const bool stream = !seg_only && C == 1 && row_bytes >= (int64_t)kStages * kStageBytes &&
+                      std::getenv("XR_NO_BULK") == nullptr;
   if (stream) {
     const int64_t min_stages = O == 1 ? kStages : 4 * kStages;  // several outputs: amortise the epilogue
     S = std::min<int64_t>(S, std::max<int64_t>(1, work / (min_stages * stage_elems)));

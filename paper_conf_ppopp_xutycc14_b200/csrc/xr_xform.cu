@@ -1,0 +1,273 @@
+// xr_xform.cu -- SURVEY.md 8(f) N1: transform-reduce, the loop body before the
+// reduction.  Two inputs x, y of the same nest:
+//   XR_XF_DISK: Monte Carlo pi (Fig 13(c) @43561-44280, section 4
+//     @42177-47503): count of x*x + y*y < 1, each operation rounded in the
+//     inputs' type with __fmul_rn / __fadd_rn (no FMA, as the paper compiles,
+//     @35389), so the predicate is decided exactly like the oracle; int64 out.
+//   XR_XF_DOT: inner product (Fig 13(b) @41386-42177): sum of x*y, dtype out.
+// Single pass like xr_reduce: private partials (16-B loads of BOTH inputs,
+// 4+4 in flight), warp shuffles, CTA smem combine, last-CTA ticket.
+// Canonical shapes R, KR, RKR (the seg decomposition) and K; column shapes
+// (RK, KRK) return XR_ERR_UNSUPPORTED.
+#include <algorithm>
+#include <cstdlib>
+
+#include "../../include/xreduce.h"
+#include "xr_internal.h"
+#include "xr_ops.cuh"
+
+namespace xr {
+
+int xform_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets);
+
+template <int XF, typename T> struct Xf;
+
+template <typename T> struct Xf<XR_XF_DISK, T> {  // count of points inside the unit disk
+  using Acc = unsigned long long;
+  using Out = long long;
+  static __device__ __forceinline__ Acc identity() { return 0ull; }
+  static __device__ __forceinline__ Acc lift(T x, T y);
+  static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return a + b; }
+  static __device__ __forceinline__ Acc lift_out(Out v) { return (Acc)v; }
+  static __device__ __forceinline__ Out finish(Acc a) { return (Out)a; }
+};
+template <> __device__ __forceinline__ unsigned long long Xf<XR_XF_DISK, float>::lift(float x, float y) {
+  return __fadd_rn(__fmul_rn(x, x), __fmul_rn(y, y)) < 1.0f ? 1ull : 0ull;
+}
+template <> __device__ __forceinline__ unsigned long long Xf<XR_XF_DISK, double>::lift(double x, double y) {
+  return __dadd_rn(__dmul_rn(x, x), __dmul_rn(y, y)) < 1.0 ? 1ull : 0ull;
+}
+
+template <typename T> __device__ __forceinline__ T mul_rn(T a, T b) { return a * b; }
+template <> __device__ __forceinline__ float mul_rn<float>(float a, float b) { return __fmul_rn(a, b); }
+template <> __device__ __forceinline__ double mul_rn<double>(double a, double b) { return __dmul_rn(a, b); }
+
+template <typename T> struct Xf<XR_XF_DOT, T> {  // inner product
+  using B = Op<OP_ADD, T>;
+  using Acc = typename B::Acc;
+  using Out = T;
+  static __device__ __forceinline__ Acc identity() { return B::identity(); }
+  static __device__ __forceinline__ Acc lift(T x, T y) {
+    if constexpr (IsFp<T>::value) return mul_rn(x, y);
+    else return B::lift(x) * B::lift(y);  // unsigned: wraps mod 2^w (C6)
+  }
+  static __device__ __forceinline__ Acc combine(Acc a, Acc b) { return B::combine(a, b); }
+  static __device__ __forceinline__ Acc lift_out(Out v) { return B::lift(v); }
+  static __device__ __forceinline__ Out finish(Acc a) { return B::finish(a); }
+};
+
+template <typename X> __device__ __forceinline__ typename X::Acc xf_warp(typename X::Acc v) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) v = X::combine(v, __shfl_xor_sync(0xffffffffu, v, off));
+  return v;
+}
+template <typename X> __device__ __forceinline__ typename X::Acc xf_block(typename X::Acc v, typename X::Acc* smem) {
+  v = xf_warp<X>(v);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (lane == 0) smem[warp] = v;
+  __syncthreads();
+  if (warp == 0) {
+    v = lane < kBlock / 32 ? smem[lane] : X::identity();
+    v = xf_warp<X>(v);
+  }
+  return v;
+}
+
+// Fold n elements of rows x, y into the lane's accumulators (group of W lanes).
+template <typename X, typename T, int W, int U>
+__device__ __forceinline__ void fold_row2(const T* __restrict__ x, const T* __restrict__ y, int64_t n, int lane,
+                                          typename X::Acc (&acc)[U][16 / sizeof(T)]) {
+  constexpr int VEC = 16 / sizeof(T);
+  if ((((uintptr_t)x ^ (uintptr_t)y) & 15u) != 0) {  // different 16-B phase: scalar lanes
+    for (int64_t i = lane; i < n; i += W) acc[0][0] = X::combine(acc[0][0], X::lift(__ldg(x + i), __ldg(y + i)));
+    return;
+  }
+  int64_t head = (int64_t)((16u - ((uint32_t)(uintptr_t)x & 15u)) & 15u) / (int64_t)sizeof(T);
+  if (head > n) head = n;
+  if (lane < head) acc[0][0] = X::combine(acc[0][0], X::lift(__ldg(x + lane), __ldg(y + lane)));
+  x += head;
+  y += head;
+  n -= head;
+  const int64_t nv = n / VEC;
+  const U128* __restrict__ xv = reinterpret_cast<const U128*>(x);
+  const U128* __restrict__ yv = reinterpret_cast<const U128*>(y);
+  int64_t v = lane;
+  for (; v + (int64_t)(U - 1) * W < nv; v += (int64_t)U * W) {
+    U128 a[U], b[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) {
+      a[k] = ld_stream(xv + v + (int64_t)k * W);
+      b[k] = ld_stream(yv + v + (int64_t)k * W);
+    }
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q)
+        acc[k][q] = X::combine(acc[k][q], X::lift(unpack<T>(a[k], q), unpack<T>(b[k], q)));
+  }
+  for (; v < nv; v += W) {
+    const U128 a = ld_stream(xv + v), b = ld_stream(yv + v);
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[0][q] = X::combine(acc[0][q], X::lift(unpack<T>(a, q), unpack<T>(b, q)));
+  }
+  const int64_t tail = n - nv * VEC;
+  if (lane < tail) acc[1 % U][0] = X::combine(acc[1 % U][0], X::lift(__ldg(x + nv * VEC + lane), __ldg(y + nv * VEC + lane)));
+}
+
+__device__ __forceinline__ int64_t xsplit(int64_t n, int64_t parts, int64_t i) {
+  const int64_t q = n / parts, r = n % parts;
+  return i * q + (i < r ? i : r);
+}
+
+// CTA-wide units, static round robin (deterministic), seg decomposition.
+template <int XF, typename T>
+__global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in2) {
+  using X = Xf<XF, T>;
+  using Acc = typename X::Acc;
+  using Out = typename X::Out;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int U = kUnroll;
+  __shared__ Acc smem[32];
+  __shared__ int s_last;
+  Out* out = static_cast<Out*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  const int64_t S = a.Sr * a.Sc;
+  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+    const int64_t o = u / S, s = u - o * S;
+    const int64_t sr = s / a.Sc, sc = s - sr * a.Sc;
+    const int64_t r0 = xsplit(a.C, a.Sr, sr), r1 = xsplit(a.C, a.Sr, sr + 1);
+    const int64_t c0 = sc == 0 ? 0 : (xsplit(a.L, a.Sc, sc) / VEC) * VEC;
+    const int64_t c1 = sc + 1 >= a.Sc ? a.L : (xsplit(a.L, a.Sc, sc + 1) / VEC) * VEC;
+    Acc acc[U][VEC];
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[k][q] = X::identity();
+    const int64_t base = o * a.oStride + c0;
+    for (int64_t r = r0; r < r1; ++r) {
+      const int64_t e = base + r * a.rowStride;
+      fold_row2<X, T, kBlock, U>(static_cast<const T*>(a.in) + e, static_cast<const T*>(in2) + e, c1 - c0,
+                                 threadIdx.x, acc);
+    }
+#pragma unroll
+    for (int k = 1; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[0][q] = X::combine(acc[0][q], acc[k][q]);
+#pragma unroll
+    for (int q = 1; q < VEC; ++q) acc[0][0] = X::combine(acc[0][0], acc[0][q]);
+    Acc v = xf_block<X>(acc[0][0], smem);
+    if (S == 1) {
+      if (threadIdx.x == 0) {
+        const Acc init = a.init_from_out ? X::lift_out(out[o]) : X::identity();
+        out[o] = X::finish(X::combine(init, v));
+      }
+    } else {
+      if (threadIdx.x == 0) {
+        partials[u] = v;
+        __threadfence();
+        s_last = (atomicAdd(&a.tickets[o], 1u) == (unsigned)(S - 1));
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        Acc w = X::identity();
+        for (int64_t i = threadIdx.x; i < S; i += kBlock) w = X::combine(w, __ldcg(partials + o * S + i));
+        w = xf_block<X>(w, smem);
+        if (threadIdx.x == 0) {
+          const Acc init = a.init_from_out ? X::lift_out(out[o]) : X::identity();
+          out[o] = X::finish(X::combine(init, w));
+          a.tickets[o] = 0u;
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+template <int XF, typename T>
+__global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const void* in2) {
+  using X = Xf<XF, T>;
+  using Out = typename X::Out;
+  Out* out = static_cast<Out*>(a.out);
+  const T* x = static_cast<const T*>(a.in);
+  const T* y = static_cast<const T*>(in2);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (int64_t)gridDim.x * blockDim.x) {
+    const typename X::Acc init = a.init_from_out ? X::lift_out(out[i]) : X::identity();
+    out[i] = X::finish(X::combine(init, a.in ? X::lift(x[i], y[i]) : X::identity()));
+  }
+}
+
+template <int XF, typename T>
+static cudaError_t xform_launch(Plan& p, const void* in2, int sms, cudaStream_t s) {
+  if (p.kernel == K_FILL || p.kernel == K_IDENT) {
+    EltArgs e = p.elt;
+    if (p.kernel == K_FILL) e.in = nullptr;
+    const int64_t grid = grid_for((e.n + kBlock - 1) / kBlock, sms, 8);
+    xform_ident_kernel<XF, T><<<(unsigned)grid, kBlock, 0, s>>>(e, in2);
+  } else {
+    static int occ = [] {
+      int n = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xform_kernel<XF, T>, kBlock, 0) != cudaSuccess || n < 1) n = 1;
+      return n;
+    }();
+    xform_kernel<XF, T><<<(unsigned)grid_for(p.units, sms, occ), kBlock, 0, s>>>(p.seg, in2);
+  }
+  count_launch();
+  return cudaPeekAtLastError();
+}
+
+}  // namespace xr
+
+using namespace xr;
+
+extern "C" int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsigned level_mask,
+                                   const void* x, const void* y, void* out, xr_stream_t stream) {
+  if (xform != XR_XF_DISK && xform != XR_XF_DOT) return XR_ERR_INVALID;
+  if (dtype < XR_INT32 || dtype > XR_FP64 || !nest_dims) return XR_ERR_INVALID;
+  if (xform == XR_XF_DISK && dtype != XR_FP32 && dtype != XR_FP64) return XR_ERR_UNSUPPORTED;
+  if ((level_mask & 7u) == 0u || (level_mask & ~(7u | XR_INIT_FROM_OUT)) != 0u) return XR_ERR_INVALID;
+  int64_t total = 1, count = 1;
+  for (int d = 0; d < 3; ++d) {
+    if (nest_dims[d] < 0) return XR_ERR_INVALID;
+    if (nest_dims[d] != 0 && total > (INT64_MAX / 8) / nest_dims[d]) return XR_ERR_INVALID;
+    total *= nest_dims[d];
+    if (!((level_mask >> d) & 1u)) count *= nest_dims[d];
+  }
+  if (count == 0) return XR_OK;
+  const int size = dtype_size(dtype), osize = xform == XR_XF_DISK ? 8 : size;
+  if (!out || (total > 0 && (!x || !y))) return XR_ERR_INVALID;
+  if (((uintptr_t)out % osize) || (total > 0 && (((uintptr_t)x % size) || ((uintptr_t)y % size))))
+    return XR_ERR_INVALID;
+  Plan p;
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  make_plan(xform == XR_XF_DOT ? XR_OP_ADD : XR_OP_LOR /* non-chain-capped */, dtype, nest_dims, level_mask & 7u,
+            0, sms, &p, /*seg_only=*/true);
+  if (p.kernel == K_NONE) return XR_OK;
+  if (p.kernel == K_COL || p.kernel == K_COLTMA) return XR_ERR_UNSUPPORTED;
+  // partial slots sized for the transform's accumulator (DISK: 8-byte counts)
+  const int64_t pbytes = p.splits > 1 ? p.units * 8 : 0;
+  void* partials = nullptr;
+  unsigned* tickets = nullptr;
+  int st = xform_workspace((cudaStream_t)stream, pbytes, p.tickets, &partials, &tickets);
+  if (st) return st;
+  const int ifo = (level_mask & XR_INIT_FROM_OUT) ? 1 : 0;
+  p.seg.in = x; p.seg.out = out; p.seg.partials = partials; p.seg.tickets = tickets; p.seg.init_from_out = ifo;
+  p.elt.in = x; p.elt.out = out; p.elt.init_from_out = ifo;
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaError_t e;
+  if (xform == XR_XF_DISK) {
+    e = dtype == XR_FP32 ? xform_launch<XR_XF_DISK, float>(p, y, sms, s) : xform_launch<XR_XF_DISK, double>(p, y, sms, s);
+  } else {
+    switch (dtype) {
+      case XR_INT32: e = xform_launch<XR_XF_DOT, int32_t>(p, y, sms, s); break;
+      case XR_INT64: e = xform_launch<XR_XF_DOT, int64_t>(p, y, sms, s); break;
+      case XR_FP32: e = xform_launch<XR_XF_DOT, float>(p, y, sms, s); break;
+      default: e = xform_launch<XR_XF_DOT, double>(p, y, sms, s); break;
+    }
+  }
+  if (e != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  return XR_OK;
+}

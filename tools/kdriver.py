@@ -98,6 +98,37 @@ def run_reduce(label, op, dtype, dims, lv, reps, timed, cache):
                           "elements_per_s": n / med * 1e3, "plan": plan}), flush=True)
 
 
+def run_xform(name, reps, timed):
+    """mc-pi-<samples log2> (fp32 pairs, disk count) or dot-rows (fp32 rows of 4096)."""
+    if name.startswith("mc-pi"):
+        n = 1 << int(name.split("-")[2]) if name.count("-") == 2 else 1 << 29
+        xf, dtype, dims, lv, byts = "disk", "fp32", (n, 1, 1), "gv", 8 * n
+    else:
+        xf, dtype, dims, lv = "dot", "fp32", (1 << 16, 1, 1 << 13), "v"
+        byts = 8 * (1 << 29)
+    n = dims[0] * dims[1] * dims[2]
+    x = tensor(n, dtype) * 2 - 1
+    y = tensor(n, dtype) * 2 - 1
+    cnt = xr.xr_out_count(dims, lv)
+    out = torch.zeros(cnt, dtype=torch.int64 if xf == "disk" else TDT[dtype], device="cuda")
+    s = torch.cuda.current_stream()
+    for _ in range(3):
+        assert xr.xr_transform_reduce(xf, dtype, dims, lv, x.data_ptr(), y.data_ptr(), out.data_ptr(), s.cuda_stream) == 0
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    for a, b in evs:
+        a.record(s)
+        xr.xr_transform_reduce(xf, dtype, dims, lv, x.data_ptr(), y.data_ptr(), out.data_ptr(), s.cuda_stream)
+        b.record(s)
+    torch.cuda.synchronize()
+    if timed:
+        ms = sorted(a.elapsed_time(b) for a, b in evs)
+        med = ms[len(ms) // 2]
+        print(json.dumps({"case": name, "dims": dims, "ms_median": med, "ms_min": ms[0], "bytes": byts,
+                          "GBps": byts / med / 1e6, "frac_of_peak": byts / med / 1e6 / peak(),
+                          "elements_per_s": n / med * 1e3}), flush=True)
+
+
 def run_heat(reps, timed, n=8192):
     t1 = torch.zeros(n * n, dtype=torch.float64, device="cuda")
     t1[:n] = 1.0
@@ -133,6 +164,9 @@ def main():
     for name in a.case:
         if name == "cfg4-heat":
             run_heat(a.reps, a.time)
+            continue
+        if name.startswith("mc-pi") or name == "dot-rows":
+            run_xform(name, a.reps, a.time)
             continue
         for c in cases(name):
             run_reduce(*c, a.reps, a.time, cache)
