@@ -140,6 +140,19 @@ typedef enum { XR_XF_DISK = 1, XR_XF_DOT = 2 } xr_xform;
 int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                         const void* x, const void* y, void* out, xr_stream_t stream);
 
+/* The paper's own code-generation scheme, an in-house A/B
+ * baseline on the same GPU: Kepler-style launch of num_gangs blocks of
+ * (vector_length x num_workers) threads (<= 0 selects the paper's 192 x (128 x
+ * 8), @35893-36486), Fig 3 loops, shared-memory interleaved log-step trees
+ * (Figs 6c, 7, 8c) and, when the gang level reduces, a global partial buffer
+ * plus a SECOND kernel launch (Fig 5c, @24887-25280; RMP @30925-31587).
+ * Masks XR_GANG, XR_WORKER, XR_VECTOR and all three (the testsuite's single-
+ * level and gang-worker-vector positions); ops + * max; dtypes int32, fp32,
+ * fp64 (Table 2).  Other combinations: XR_ERR_UNSUPPORTED.  Same output
+ * layout and init semantics as xr_reduce.  Two launches when gang reduces. */
+int xr_reduce_paper(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask, const void* in,
+                    void* out, int num_gangs, int num_workers, int vector_length, xr_stream_t stream);
+
 /* ------------------------------------------------------------ planning ---- */
 
 /* Canonical shapes after dropping extent-1 levels and merging adjacent levels

@@ -92,6 +92,7 @@ _SIGS = {
     "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
     "xr_transform_reduce": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
+    "xr_reduce_paper": (_c, [_c, _c, _i64p, _u, _vp, _vp, _c, _c, _c, _vp]),
     "xr_heat_step_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded_sim": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _c, ctypes.POINTER(_vp),
@@ -195,6 +196,13 @@ def xr_reduce_sharded_sim(op, dtype, local_dims, level_mask, shard_ptrs, out_ptr
 
 
 XFORMS = {"disk": 1, "dot": 2}
+
+
+def xr_reduce_paper(op, dtype, nest_dims, level_mask, in_ptr: int, out_ptr: int, num_gangs: int = 0,
+                    num_workers: int = 0, vector_length: int = 0, stream: int = 0) -> int:
+    """The paper's own scheme (A/B baseline, include/xreduce.h)."""
+    return _lib.xr_reduce_paper(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask), in_ptr or None,
+                                out_ptr or None, num_gangs, num_workers, vector_length, stream or None)
 
 
 def xr_transform_reduce(xform, dtype, nest_dims, level_mask, x_ptr: int, y_ptr: int, out_ptr: int,

@@ -420,6 +420,17 @@ int xform_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partia
   *tickets = w.tickets;
   return XR_OK;
 }
+// used by xr_paper.cu: the partial / RMP buffers of the paper-faithful kernels
+int paper_workspace(cudaStream_t s, int64_t bytes, void** buf) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  std::lock_guard<std::mutex> lock(g_mu);
+  Workspace& w = g_ws[{dev, (uintptr_t)s}];
+  int st = ensure_ws(w, bytes, 0, s);
+  if (st) return st;
+  *buf = w.partials;
+  return XR_OK;
+}
 // used by xr_heat.cu: the same per-(device, stream) workspace
 int heat_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets) {
   int dev = 0;
