@@ -21,5 +21,7 @@ def _built():
     import __graft_entry__
     datagen.build()
     oracle.build()
-    __graft_entry__._native().build()  # libxreduce.so (no-op when up to date)
+    nat = __graft_entry__._native()
+    nat.build()              # libxreduce.so (no-op when up to date)
+    nat.build_devapi_test()  # tests/devapi/libxr_devapi_test.so
     yield

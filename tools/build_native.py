@@ -38,7 +38,8 @@ def _sources():
     cu = sorted(f for f in os.listdir(CSRC) if f.endswith(".cu"))
     cpp = sorted(f for f in os.listdir(CSRC) if f.endswith(".cpp"))
     hdr = [os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".h", ".cuh"))]
-    hdr.append(os.path.join(ROOT, "include", "xreduce.h"))
+    inc = os.path.join(ROOT, "include")
+    hdr += [os.path.join(inc, f) for f in os.listdir(inc)]
     return cu, cpp, hdr
 
 
@@ -93,5 +94,22 @@ def build(force: bool = False, ptxas_verbose: bool = False, quiet: bool = True) 
     return SO
 
 
+def build_devapi_test(force: bool = False) -> str:
+    """tests/devapi/libxr_devapi_test.so: a TEST module that uses only the
+    public device header include/xreduce_device.cuh."""
+    src = os.path.join(ROOT, "tests", "devapi", "devapi_test.cu")
+    so = os.path.join(ROOT, "tests", "devapi", "libxr_devapi_test.so")
+    deps = [src] + [os.path.join(ROOT, "include", f) for f in os.listdir(os.path.join(ROOT, "include"))]
+    if force or _stale(so, deps):
+        cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
+               "--expt-relaxed-constexpr", src, "-o", so, "-cudart", "static"]
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            sys.stderr.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
+            raise RuntimeError("devapi test build failed")
+    return so
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, ptxas_verbose="--ptxas-v" in sys.argv, quiet=False))
+    print(build_devapi_test(force="--force" in sys.argv))
