@@ -140,6 +140,24 @@ typedef enum { XR_XF_DISK = 1, XR_XF_DOT = 2 } xr_xform;
 int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                         const void* x, const void* y, void* out, xr_stream_t stream);
 
+/* Several reduction variables with mixed dtypes in ONE pass (
+ * PAPER.md 3.3 @31605-32570: one reduction clause with e.g. an int and a float
+ * variable sharing one shared-memory pool sized for the largest type).  Each
+ * variable has its own op, dtype, input (DEVICE, n0*n1*n2 elements) and output
+ * (DEVICE, xr_out_count elements); all share nest_dims and level_mask (with
+ * XR_INIT_FROM_OUT applying to every output).  1 <= nvars <= 8.  Semantics per
+ * variable exactly as xr_reduce; no output may overlap an input or another
+ * output.  Canonical shapes R, KR, RKR, K and empty reduced extents are
+ * supported; column shapes (RK, KRK) return XR_ERR_UNSUPPORTED.  One launch. */
+typedef struct {
+  int op;          /* xr_op   */
+  int dtype;       /* xr_dtype */
+  const void* in;
+  void* out;
+} xr_var;
+int xr_reduce_multi(int nvars, const xr_var* vars, const int64_t nest_dims[3], unsigned level_mask,
+                    xr_stream_t stream);
+
 /* The paper's own code-generation scheme, an in-house A/B
  * baseline on the same GPU: Kepler-style launch of num_gangs blocks of
  * (vector_length x num_workers) threads (<= 0 selects the paper's 192 x (128 x

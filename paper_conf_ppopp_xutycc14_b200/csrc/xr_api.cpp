@@ -420,6 +420,10 @@ int xform_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partia
   *tickets = w.tickets;
   return XR_OK;
 }
+// used by xr_multi.cu: the same per-(device, stream) workspace
+int multi_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partials, unsigned** tickets) {
+  return xform_workspace(s, pbytes, ntick, partials, tickets);
+}
 // used by xr_paper.cu: the partial / RMP buffers of the paper-faithful kernels
 int paper_workspace(cudaStream_t s, int64_t bytes, void** buf) {
   int dev = 0;
