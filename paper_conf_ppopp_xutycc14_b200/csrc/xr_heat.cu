@@ -236,6 +236,7 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
         if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
         if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
       }
+      fence_proxy_async_smem();  // generic reads before the async refill
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[(r - 1) % kHeatSlots]);  // row r-1 is dead for this warp
     }

@@ -379,6 +379,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
           for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x, q)));
         }
       }
+      fence_proxy_async_smem();  // generic reads before the async refill
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[slot]);  // this warp is done with the stage
     }
@@ -536,6 +537,7 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
           }
         }
       }
+      fence_proxy_async_smem();  // generic reads before the async refill
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[slot]);  // the stage is consumed into registers
 #pragma unroll
@@ -796,6 +798,7 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
           for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
         }
       }
+      fence_proxy_async_smem();  // generic reads before the async refill
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[slot]);
     }

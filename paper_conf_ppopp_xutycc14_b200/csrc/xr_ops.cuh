@@ -91,6 +91,12 @@ constexpr int kConsWarps = 8;
 constexpr int kConsThreads = 32 * kConsWarps;
 constexpr int kWsBlock = kConsThreads + 32;  // + the producer warp
 
+// Order this thread's generic-proxy shared-memory accesses before later
+// async-proxy (bulk copy / TMA) accesses to the same memory: a consumer
+// executes it before releasing a ring stage that the producer will refill.
+__device__ __forceinline__ void fence_proxy_async_smem() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
 }

@@ -313,3 +313,25 @@ def test_rows_kernel_short_rows(dtype, row_bytes):
         check(op, dtype, dims, "v", gpu_reduce(op, dtype, dims, "v", x, init=init), x, init=init)
         if O >= 1003 and row_bytes <= 2048:
             assert plan["kernel"] == "rows"
+
+
+def test_ring_kernels_stress_repeatable():
+    """The bulk/TMA ring kernels (stream, rows, coltma, heat) reuse shared-memory
+    stages released through mbarriers; a real write-after-read race would
+    corrupt results nondeterministically.  Integer results must be identical to
+    the oracle on every one of many back-to-back runs (compute-sanitizer
+    racecheck cannot model mbarrier/async-proxy ordering, profiles/)."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    cases = [("+", "int32", (1 << 22, 1, 1), "gwv"), ("^", "int64", (64, 1, 1 << 15), "v"),
+             ("+", "int32", (8192, 1, 512), "v"), ("|", "int32", (4096, 1, 2048), "g")]
+    for op, dtype, dims, lv in cases:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, 77)
+        ref = oracle.reduce(op, dtype, dims, lv, x)
+        xd = torch.from_numpy(x).cuda()
+        outs = [torch.empty(ref.size, dtype=xd.dtype, device="cuda") for _ in range(50)]
+        for o in outs:  # back to back on one stream: stages are refilled under load
+            assert xr.xr_reduce(op, dtype, dims, lv, xd.data_ptr(), o.data_ptr()) == 0
+        torch.cuda.synchronize()
+        for o in outs:
+            assert np.array_equal(o.cpu().numpy(), ref), (op, dtype, dims, lv)

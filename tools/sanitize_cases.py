@@ -1,0 +1,59 @@
+#!/usr/bin/env python3
+"""Small invocations of every kernel family, for compute-sanitizer
+(memcheck / racecheck / synccheck / initcheck).  Exits non-zero on a parity error."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import oracle  # noqa: E402  (test infrastructure: checks the results)
+import paper_conf_ppopp_xutycc14_b200 as xr  # noqa: E402
+from datagen import recipes  # noqa: E402
+from gpu_util import check, gpu_reduce  # noqa: E402
+
+cases = [
+    ("+", "fp32", (1 << 18, 1, 1), "gwv"),        # stream (R)
+    ("max", "int32", (64, 1, 1 << 14), "v"),      # stream (KR, 64 KiB rows)
+    ("+", "fp32", (300, 1, 512), "v"),            # rows kernel
+    ("^", "int64", (37, 41, 123), "v"),           # seg W=32
+    ("*", "int32", (5, 3, 31), "v"),              # seg W=8
+    ("+", "fp64", (40, 33, 700), "gv"),           # seg RKR split
+    ("&&", "fp32", (700, 1, 512), "g"),           # coltma
+    ("min", "fp32", (999, 1, 33), "g"),           # col (unaligned)
+    ("|", "int32", (20, 300, 64), "w"),           # col KRK
+    ("+", "int32", (3, 1, 5), "w"),               # ident
+]
+for op, dtype, dims, lv in cases:
+    x = recipes.make({"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "^": "bxor", "&&": "land",
+                      "|": "bor"}[op], dims, oracle.mask_of(lv), dtype, 1)
+    check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
+# heat (bulk + register variants), transform-reduce, multi, paper kernels
+for nj, ni in [(70, 1030), (33, 67)]:
+    T0 = oracle.heat_init(nj, ni)
+    t1 = torch.from_numpy(T0).cuda()
+    t2 = t1.clone()
+    res = torch.zeros(3, dtype=torch.float64, device="cuda")
+    assert xr.xr_heat_run(nj, ni, 3, t1.data_ptr(), t2.data_ptr(), res.data_ptr()) == 0
+    torch.cuda.synchronize()
+    assert res.cpu().tolist() == oracle.heat(nj, ni, 3, T0)[1].tolist()
+xs = torch.rand(1 << 16, device="cuda") * 2 - 1
+ys = torch.rand(1 << 16, device="cuda") * 2 - 1
+cnt = torch.zeros(1, dtype=torch.int64, device="cuda")
+assert xr.xr_transform_reduce("disk", "fp32", (1 << 16, 1, 1), "gwv", xs.data_ptr(), ys.data_ptr(), cnt.data_ptr()) == 0
+torch.cuda.synchronize()
+assert int(cnt.item()) == int(oracle.transform_reduce("disk", "fp32", (1 << 16, 1, 1), "gwv",
+                                                      xs.cpu().numpy(), ys.cpu().numpy())[0])
+o1 = torch.zeros(64, device="cuda")
+o2 = torch.zeros(64, dtype=torch.int32, device="cuda")
+xi = torch.arange(64 * 1000, dtype=torch.int32, device="cuda")
+assert xr.xr_reduce_multi([("+", "fp32", xs.data_ptr(), o1.data_ptr()), ("max", "int32", xi.data_ptr(), o2.data_ptr())],
+                          (64, 1, 1000), "v") == 0
+pz = torch.zeros(64 * 32, device="cuda")
+assert xr.xr_reduce_paper("+", "fp32", (8, 8, 1000), "w", xs.data_ptr(), pz.data_ptr(), 16, 8, 128) == 0
+assert xr.xr_reduce_paper("+", "fp32", (8, 8, 1000), "gwv", xs.data_ptr(), pz.data_ptr(), 16, 8, 128) == 0
+torch.cuda.synchronize()
+print("sanitize cases OK")
