@@ -16,6 +16,7 @@ constexpr int kUnitsPerCta = 8;      // dynamic units per resident CTA (tail bal
 enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6, K_ROWS = 7 };
 
 constexpr int kStages = 4;          // bulk-copy ring depth (stream kernel)
+constexpr int64_t kSmallBytes = int64_t(16) << 20;  // below: register kernels (latency bound)
 constexpr int kStageBytes = 16384;  // bytes per stage
 
 // Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]

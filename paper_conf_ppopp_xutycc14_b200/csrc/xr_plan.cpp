@@ -37,6 +37,7 @@ int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
                int num_sms, Plan* p, bool seg_only) {
   *p = Plan();
+  bool seg_only_small = false;
   const int size = dtype_size(dtype);
   const int vec = 16 / size;
   const int asz = acc_size(op, dtype);
@@ -81,6 +82,16 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     }
   }
   for (int r = 0; r < nr; ++r) p->cdims[r] = run_n[r];
+  // Small inputs are latency bound, not bandwidth bound: the staged (bulk /
+  // TMA ring) kernels would run on a few dozen CTAs, so below kSmallBytes the
+  // register kernels, which spread one load round over many CTAs, are used.
+  {
+    int64_t total = 1;
+    for (int d = 0; d < 3; ++d) total *= dims[d];
+    const char* env = std::getenv("XR_SMALL_BYTES");  // test / tuning override
+    const int64_t small = env ? std::atoll(env) : kSmallBytes;
+    if (total * size < small) seg_only_small = true;
+  }
 
   // (3) the pattern
   if (nr == 0 || (nr == 1 && !run_red[0])) {  // K: every reduced extent is 1
@@ -105,7 +116,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       return;
     }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
-    if (aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
+    if (!seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {
       const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
       const int64_t tiles = cdiv(K, TWt);
@@ -155,6 +166,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int64_t base = B * tiles;
     if (base < kUnitsPerCta * target_ctas) {
       S = cdiv(kUnitsPerCta * target_ctas, base);
+      // >= 4 load rounds per warp: on small inputs a split's extra ticket round
+      // costs more than its parallelism buys (cfg1 G/W: 4.0 us unsplit vs 5.4 us)
       S = std::min<int64_t>(S, std::max<int64_t>(1, R / (4 * NW * kUnroll)));
       S = std::min<int64_t>(S, 128);  // the last CTA of a tile folds S rows (8 warps x 4 loads)
     }
@@ -184,7 +197,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   const int64_t row_bytes = L * size;
   // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
   // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
-  if (!seg_only && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 && (row_bytes & (row_bytes - 1)) == 0 &&
+  if (!seg_only && !seg_only_small && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 &&
+      (row_bytes & (row_bytes - 1)) == 0 &&
       in_addr % 16 == 0 && std::getenv("XR_NO_BULK") == nullptr) {
     const int64_t rps = kStageBytes / row_bytes;
     const int64_t nst = cdiv(O, rps);
@@ -212,12 +226,14 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   int64_t S = 1;
   if (O < want_units) {
     S = cdiv(want_units, O);
-    S = std::min<int64_t>(S, std::max<int64_t>(1, work / (4 * min_unit_elems(W))));
+    // register path: one unrolled load round per thread is enough (small,
+    // latency-bound inputs get many CTAs); the stream path re-caps below
+    S = std::min<int64_t>(S, std::max<int64_t>(1, work / min_unit_elems(W)));
   }
   // long contiguous rows (R, KR): the bulk-copy stream kernel; every unit must
   // cover at least kStages stages so the producer stays <= 3 units ahead
   const int64_t stage_elems = kStageBytes / size;
-  const bool stream = !seg_only && C == 1 && row_bytes >= (int64_t)kStages * kStageBytes &&
+  const bool stream = !seg_only && !seg_only_small && C == 1 && row_bytes >= (int64_t)kStages * kStageBytes &&
                       std::getenv("XR_NO_BULK") == nullptr;
   if (stream) {
     const int64_t min_stages = O == 1 ? kStages : 4 * kStages;  // several outputs: amortise the epilogue
