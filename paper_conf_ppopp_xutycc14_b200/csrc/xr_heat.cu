@@ -28,6 +28,7 @@ int heat_workspace(cudaStream_t s, int64_t pbytes, int64_t ntick, void** partial
 
 constexpr int kHeatRows = 64;     // rows marched per warp (halo re-read: 2/64)
 constexpr int kHeatPrefetch = 4;  // rows in flight per lane
+constexpr int kHeatRowsPersistent = 12;  // output rows per tile of the persistent kernel
 
 struct HeatArgs {
   const double* T1;
@@ -263,6 +264,152 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
   }
 }
 
+// Persistent variant of the bulk sweep: grid = resident CTAs; the producer
+// warp claims tiles (row-block-major, so the halo rows shared by vertically
+// adjacent tiles are re-read from L2) from a device counter and streams their
+// rows through the ring WITHOUT draining between tiles; consumers release
+// every row slot exactly once (row r-1 after output row r, the last two rows
+// at the end of a tile).  Removes wave quantisation (2048 tiles on ~740
+// resident CTAs) and the per-CTA fill / drain of the one-tile version.  The
+// max residual is exact, so the result does not depend on tile assignment.
+struct HeatPArgs {
+  HeatArgs h;
+  int64_t gx, gy;               // column tiles, row blocks
+  unsigned long long* sched;    // [2] tile counter + exit counter
+};
+
+__global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa) {
+  using O = Op<OP_MAX, double>;
+  constexpr int RING = 8;
+  __shared__ __align__(128) double slots[kHeatSlots][kSlotDoubles];
+  __shared__ __align__(8) uint64_t full[kHeatSlots];
+  __shared__ __align__(8) uint64_t empty[kHeatSlots];
+  __shared__ long long s_tiles[RING];
+  __shared__ double smem[32];
+  __shared__ int s_last;
+  const HeatArgs& a = pa.h;
+  const int tid0 = threadIdx.x, warp = tid0 >> 5, lane = tid0 & 31;
+  const int64_t ni = a.ni, ntiles = pa.gx * pa.gy;
+  auto tile_geom = [&](long long t, int64_t* c0, int64_t* j0, int64_t* j1) {
+    const int64_t ty = t / pa.gx, tx = t - ty * pa.gx;  // row-block-major
+    *c0 = tx * kTileCols;
+    *j0 = a.jb + ty * a.rows;
+    *j1 = min(*j0 + a.rows, a.je);
+  };
+  if (tid0 == 0) {
+    for (int k = 0; k < kHeatSlots; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+  if (warp == 0) {  // ---------------- producer warp
+    if (lane == 0) {
+      int64_t q = 0;  // global row counter (slot = q % kHeatSlots)
+      int seq = 0;
+      long long t = (long long)atomicAdd(pa.sched, 1ull);
+      while (true) {
+        const long long nt = (long long)atomicAdd(pa.sched, 1ull);
+        const int slot0 = (int)(q % kHeatSlots);
+        s_tiles[seq & (RING - 1)] = t < ntiles ? t : -1;
+        ++seq;
+        if (t >= ntiles) {
+          if (q >= kHeatSlots) mbar_wait(&empty[slot0], (unsigned)(((q / kHeatSlots) - 1) & 1));
+          mbar_arrive(&full[slot0]);
+          break;
+        }
+        int64_t c0, j0, j1;
+        tile_geom(t, &c0, &j0, &j1);
+        const int64_t ws = max(c0 - 2, (int64_t)0), we = min(c0 + kTileCols + 2, ni);
+        const unsigned wbytes = (unsigned)((we - ws) * 8);
+        const int64_t soff = ws - (c0 - 2);
+        for (int64_t r = 0; r < j1 - j0 + 2; ++r, ++q) {  // rows j0-1 .. j1
+          const int slot = (int)(q % kHeatSlots);
+          if (q >= kHeatSlots) mbar_wait(&empty[slot], (unsigned)(((q / kHeatSlots) - 1) & 1));
+          mbar_expect_tx(&full[slot], wbytes);
+          bulk_g2s(&slots[slot][soff], a.T1 + (j0 - 1 + r) * ni + ws, wbytes, &full[slot]);
+        }
+        t = nt;
+      }
+      sched_exit(pa.sched);
+    }
+    return;
+  }
+  // ---------------- consumer warps
+  const int tid = tid0 - 32, cw = warp - 1;
+  double err = 0.0;
+  int seq = 0;
+  int64_t q = 0;  // global row counter, as the producer's
+  while (true) {
+    mbar_wait(&full[q % kHeatSlots], (unsigned)((q / kHeatSlots) & 1));  // first row of the tile
+    const long long t = s_tiles[seq & (RING - 1)];
+    ++seq;
+    if (t < 0) break;
+    int64_t c0, j0, j1;
+    tile_geom(t, &c0, &j0, &j1);
+    const int64_t nrows = j1 - j0 + 2;
+    const int64_t qb = q;  // global index of row 0 of this tile
+    mbar_wait(&full[(qb + 1) % kHeatSlots], (unsigned)(((qb + 1) / kHeatSlots) & 1));
+    const int64_t col = c0 + 2 * tid;
+    const int li = 2 + 2 * tid;
+    const bool i0 = col >= 1 && col <= ni - 2;
+    const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
+    for (int64_t r = 1; r < nrows - 1; ++r) {
+      const int64_t qd = qb + r + 1;
+      mbar_wait(&full[qd % kHeatSlots], (unsigned)((qd / kHeatSlots) & 1));
+      if (i0 || i1) {
+        const double* up = slots[(qb + r - 1) % kHeatSlots];
+        const double* cur = slots[(qb + r) % kHeatSlots];
+        const double* dn = slots[qd % kHeatSlots];
+        const double2 u2 = *reinterpret_cast<const double2*>(up + li);
+        const double2 c2 = *reinterpret_cast<const double2*>(cur + li);
+        const double2 d2 = *reinterpret_cast<const double2*>(dn + li);
+        const double l = cur[li - 1], rr = cur[li + 2];
+        const double n0 = stencil(u2.x, d2.x, l, c2.y);
+        const double n1 = stencil(u2.y, d2.y, c2.x, rr);
+        double* dst = a.T2 + (j0 + r - 1) * ni + col;
+        if (i0 && i1) {
+          __stcs(reinterpret_cast<double2*>(dst), make_double2(n0, n1));
+        } else if (i0) {
+          __stcs(dst, n0);
+        } else {
+          __stcs(dst + 1, n1);
+        }
+        if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
+        if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
+      }
+      fence_proxy_async_smem();  // generic reads before the async refill
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[(qb + r - 1) % kHeatSlots]);  // row r-1 is dead
+    }
+    fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {  // the tile's last two rows
+      mbar_arrive(&empty[(qb + nrows - 2) % kHeatSlots]);
+      mbar_arrive(&empty[(qb + nrows - 1) % kHeatSlots]);
+    }
+    q = qb + nrows;
+  }
+  err = cons_reduce<OP_MAX, double>(err, smem, cw, lane);
+  if (tid == 0) {
+    a.partials[blockIdx.x] = err;
+    __threadfence();
+    s_last = (atomicAdd(a.tickets, 1u) == gridDim.x - 1u);
+  }
+  cons_sync();
+  if (s_last) {
+    __threadfence();
+    double w = 0.0;
+    for (int64_t k = tid; k < gridDim.x; k += kConsThreads) w = O::combine(w, ld_partial(a.partials + k));
+    w = cons_reduce<OP_MAX, double>(w, smem, cw, lane);
+    if (tid == 0) {
+      *a.residual = w;
+      *a.tickets = 0u;
+    }
+  }
+}
+
 // Sweep output rows [jb, je) of an nj x ni buffer (rows jb-1 and je are read).
 static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
                        double* residual, cudaStream_t s) {
@@ -270,9 +417,15 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   const bool bulk = v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr;
   const int strip = bulk ? kTileCols : 32 * (v2 ? 2 : 1) * (kBlock / 32);
   const int64_t gx = (ni + strip - 1) / strip;
-  // 64-row tiles (2048 CTAs at 8192^2).  Sizing row blocks for one full wave
-  // of resident CTAs measured slower (0.79 vs 0.89 of peak, r01), so it is not used.
-  const int64_t rows = kHeatRows;
+  // 64-row tiles (one tile per CTA: 2048 CTAs at 8192^2; the persistent kernel
+  // claims them dynamically).  Sizing row blocks for one full wave of resident
+  // one-tile CTAs measured slower (0.79 vs 0.89 of peak, r01).
+  // The persistent bulk kernel balances best with short tiles (r01 sweep at
+  // 8192^2: 8 rows 0.908, 12 rows 0.929, 16 rows 0.918, 64 rows 0.869 of peak;
+  // halo rows come from L2).
+  const char* hr = std::getenv("XR_HEAT_ROWS");  // tuning override
+  const bool persistent = bulk && std::getenv("XR_HEAT_ONE_TILE") == nullptr;
+  const int64_t rows = hr ? std::max(4, std::atoi(hr)) : (persistent ? kHeatRowsPersistent : kHeatRows);
   const int64_t gy = je > jb ? (je - jb + rows - 1) / rows : 1;
   if (gy > 65535) return XR_ERR_INVALID;
   HeatArgs a;
@@ -281,12 +434,29 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   a.jb = jb; a.je = je;
   void* partials = nullptr;
   unsigned* tickets = nullptr;
-  int st = heat_workspace(s, a.ntiles * (int64_t)sizeof(double), 1, &partials, &tickets);
+  int st = heat_workspace(s, a.ntiles * (int64_t)sizeof(double), 6, &partials, &tickets);  // ticket + 2 x u64
   if (st) return st;
   a.partials = static_cast<double*>(partials);
   a.tickets = tickets;
   dim3 grid((unsigned)gx, (unsigned)gy);
-  if (bulk) heat_bulk_kernel<<<grid, kWsBlock, 0, s>>>(a);
+  const char* hp = std::getenv("XR_HEAT_ONE_TILE");  // A/B: one tile per CTA
+  if (bulk && hp == nullptr && je > jb) {
+    static int occ = [] {
+      int n = 0;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, heat_persistent_kernel, kWsBlock, 0) != cudaSuccess || n < 1)
+        n = 1;
+      return n;
+    }();
+    int dev = 0, sms = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    HeatPArgs pa;
+    pa.h = a;
+    pa.gx = gx;
+    pa.gy = gy;
+    pa.sched = reinterpret_cast<unsigned long long*>(tickets + 2);  // after the residual ticket (8-B aligned)
+    const int64_t pgrid = std::min<int64_t>(gx * gy, (int64_t)sms * occ);
+    heat_persistent_kernel<<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
+  } else if (bulk) heat_bulk_kernel<<<grid, kWsBlock, 0, s>>>(a);
   else if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
   else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);
   count_launch();

@@ -143,20 +143,6 @@ __device__ __forceinline__ typename Op<OP, T>::Acc fold_partials(const typename 
   return w;
 }
 
-// Dynamic unit claiming for CTA-wide work: thread 0 fetches the next unit
-// index (prefetched one unit ahead into a parity slot) from a device counter;
-// the last CTA to exit resets the counters for the next launch.
-__device__ __forceinline__ void sched_exit(unsigned long long* c) {
-  if (threadIdx.x == 0) {
-    __threadfence();
-    const unsigned long long t = atomicAdd(c + 1, 1ull);
-    if (t == (unsigned long long)gridDim.x - 1ull) {
-      c[0] = 0ull;
-      c[1] = 0ull;
-    }
-  }
-}
-
 // ------------------------------------------------------------- seg kernel
 // Groups of W lanes (8 or 32: inside a warp; W == BLOCK: the whole CTA) each
 // reduce work units; a unit is (output o, split s).  Splits (S > 1) only

@@ -119,3 +119,20 @@ __device__ __forceinline__ typename Op<OP, T>::Acc cons_reduce(typename Op<OP, T
   return v;
 }
 }  // namespace xr
+
+namespace xr {
+// Dynamic unit claiming for CTA-wide work: thread 0 fetches the next unit
+// index (prefetched one unit ahead into a parity slot) from a device counter;
+// the last CTA to exit resets the counters for the next launch.
+__device__ __forceinline__ void sched_exit(unsigned long long* c) {
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long t = atomicAdd(c + 1, 1ull);
+    if (t == (unsigned long long)gridDim.x - 1ull) {
+      c[0] = 0ull;
+      c[1] = 0ull;
+    }
+  }
+}
+
+}  // namespace xr
