@@ -542,6 +542,164 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
   }
 }
 
+// ------------------------------------------------------------- flat column kernel
+// RK / KRK with NARROW rows (row_bytes = K*size a power of two in [16, 4096] B,
+// 16-B aligned): a CTA's load round (256 threads x 16 B = 4 KiB) covers whole
+// rows, so thread t always meets the same column group (t*16 mod row_bytes)
+// and a unit -- a block of whole rows of one batch -- is ONE contiguous range,
+// streamed with fully coalesced 16-B loads (4 in flight per thread).  The
+// worker tier folds the threads of each column group in shared memory (fixed
+// order); the gang tier is the two-level ticket of coltma (unit partial rows
+// of K values -> groups of kGroupFold -> batch).  The register column kernel
+// left 1/2 to 31/32 of its lanes idle on such rows (r01: 1 TB/s on the
+// paper's 2^20 x 2 x 32 gang case).
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) colflat_kernel(ColArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int U = kUnroll;
+  __shared__ Acc red[kBlock][VEC];
+  __shared__ int s_last;
+  const int t = threadIdx.x;
+  const int64_t row_bytes = a.K * (int64_t)sizeof(T);
+  const int G = (int)(row_bytes >> 4);            // 16-B column groups per row (1..256)
+  const int64_t rp4k = 4096 / row_bytes;           // rows per 4 KiB load round
+  const int64_t nblk = (a.R + rp4k - 1) / rp4k;    // 4 KiB row blocks per batch
+  T* out = static_cast<T*>(a.out);
+  Acc* partials = static_cast<Acc*>(a.partials);
+  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x) {
+    const int64_t b = u / a.S, s = u - b * a.S;
+    const int64_t r0 = min(split_lo(nblk, a.S, s) * rp4k, a.R), r1 = min(split_lo(nblk, a.S, s + 1) * rp4k, a.R);
+    const U128* __restrict__ base = reinterpret_cast<const U128*>(static_cast<const T*>(a.in) + (b * a.R + r0) * a.K);
+    const int64_t nv = (r1 - r0) * (row_bytes >> 4);  // 16-B vectors of the unit
+    Acc acc[U][VEC];
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[k][q] = O::identity();
+    int64_t v = t;
+    for (; v + (int64_t)(U - 1) * kBlock < nv; v += (int64_t)U * kBlock) {
+      U128 x[U];
+#pragma unroll
+      for (int k = 0; k < U; ++k) x[k] = ld_stream(base + v + (int64_t)k * kBlock);
+#pragma unroll
+      for (int k = 0; k < U; ++k)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
+    }
+    for (; v < nv; v += kBlock) {
+      const U128 x = ld_stream(base + v);
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], O::lift(unpack<T>(x, q)));
+    }
+#pragma unroll
+    for (int k = 1; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], acc[k][q]);
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) red[t][q] = acc[0][q];
+    __syncthreads();
+    // a3: column group g (< G) folds threads g, g+G, g+2G, ... in order; the
+    // K = G*VEC unit results go to smem row red[0..G)
+    Acc w[VEC];
+    if (t < G) {
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) w[q] = red[t][q];
+      for (int m = t + G; m < kBlock; m += G)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) w[q] = O::combine(w[q], red[m][q]);
+    }
+    __syncthreads();
+    if (t < G) {
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) reinterpret_cast<Acc*>(red)[t * VEC + q] = w[q];
+    }
+    __syncthreads();
+    const Acc* col = reinterpret_cast<const Acc*>(red);  // col[c], c < K
+    if (a.S == 1) {
+      for (int c = t; c < a.K; c += kBlock) out[b * a.K + c] = merge_init<OP, T>(col[c], out, b * a.K + c, a.init_from_out);
+    } else {
+      // a4, two levels over the S unit partial rows of batch b (K values each)
+      Acc* P1 = partials + b * a.S * a.K;                         // [S][K]
+      Acc* P2 = partials + a.B * a.S * a.K + b * a.G2 * a.K;      // [G2][K]
+      unsigned* gt = a.tickets + b * a.G2;
+      unsigned* tt = a.tickets + a.B * a.G2 + b;
+      const int64_t gi = s / kGroupFold, g0 = gi * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
+      // fold rows [0, n) of a [n][K] partial block into column c; when K < the
+      // CTA, kBlock / K row phases fold in parallel and meet in shared memory
+      Acc* redf = reinterpret_cast<Acc*>(red);  // >= kBlock slots
+      auto fold_rows = [&](const Acc* src, int64_t n, auto&& emit) {
+        if (a.K < kBlock) {
+          const int K = (int)a.K, nph = kBlock / K, c = t % K, ph = t / K;
+          Acc z = O::identity();
+          int64_t r = ph;
+          for (; r + 3 * nph < n; r += 4 * nph) {
+            Acc y[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) y[k] = ld_partial(src + (r + k * nph) * a.K + c);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) z = O::combine(z, y[k]);
+          }
+          for (; r < n; r += nph) z = O::combine(z, ld_partial(src + r * a.K + c));
+          __syncthreads();  // redf may still be read (col) by other threads
+          redf[ph * K + c] = z;
+          __syncthreads();
+          if (t < K) {
+            Acc w2 = O::identity();
+            for (int p2 = 0; p2 < nph; ++p2) w2 = O::combine(w2, redf[p2 * K + t]);
+            emit(t, w2);
+          }
+        } else {
+          for (int c = t; c < a.K; c += kBlock) {
+            Acc z = O::identity();
+            int64_t r = 0;
+            for (; r + 3 < n; r += 4) {
+              Acc y[4];
+#pragma unroll
+              for (int k = 0; k < 4; ++k) y[k] = ld_partial(src + (r + k) * a.K + c);
+#pragma unroll
+              for (int k = 0; k < 4; ++k) z = O::combine(z, y[k]);
+            }
+            for (; r < n; ++r) z = O::combine(z, ld_partial(src + r * a.K + c));
+            emit(c, z);
+          }
+        }
+      };
+      for (int c = t; c < a.K; c += kBlock) P1[s * a.K + c] = col[c];
+      __syncthreads();
+      if (t == 0) {
+        __threadfence();
+        s_last = (atomicAdd(&gt[gi], 1u) == (unsigned)(gsz - 1));
+      }
+      __syncthreads();
+      if (s_last) {
+        __threadfence();
+        auto to_out = [&](int c, Acc z) { out[b * a.K + c] = merge_init<OP, T>(z, out, b * a.K + c, a.init_from_out); };
+        if (a.G2 == 1) {
+          fold_rows(P1 + g0 * a.K, gsz, to_out);
+          if (t == 0) gt[gi] = 0u;
+        } else {
+          fold_rows(P1 + g0 * a.K, gsz, [&](int c, Acc z) { P2[gi * a.K + c] = z; });
+          __syncthreads();
+          if (t == 0) {
+            gt[gi] = 0u;
+            __threadfence();
+            s_last = (atomicAdd(tt, 1u) == (unsigned)(a.G2 - 1));
+          }
+          __syncthreads();
+          if (s_last) {
+            __threadfence();
+            fold_rows(P2, a.G2, to_out);
+            if (t == 0) *tt = 0u;
+          }
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // ------------------------------------------------------------- col kernel
 // Lanes own VEC contiguous kept columns (a 32*VEC-column tile per warp row);
 // the CTA's warps stride over the reduced rows of a row chunk; the worker tier
@@ -971,6 +1129,11 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.seg);
+      break;
+    }
+    case K_COLFLAT: {
+      static int occ = occupancy(colflat_kernel<OP, T>, kBlock);
+      colflat_kernel<OP, T><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
       break;
     }
     case K_COLTMA: {

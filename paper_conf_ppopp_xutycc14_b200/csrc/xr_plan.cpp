@@ -115,6 +115,39 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       p->kernel = K_COL;
       return;
     }
+    // Narrow rows (power-of-two row_bytes in [16, 512] B, or up to 4 KiB for
+    // small inputs): the flat column kernel streams whole rows contiguously.
+    const int64_t row_bytes = K * size;
+    const bool pow2 = (row_bytes & (row_bytes - 1)) == 0;
+    if (aligned && pow2 && row_bytes >= 16 &&
+        (row_bytes <= 512 || (seg_only_small && row_bytes <= 4096)) && std::getenv("XR_NO_FLAT") == nullptr) {
+      const int64_t rp4k = 4096 / row_bytes;
+      const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch
+      const char* eu = std::getenv("XR_FLAT_UNITS_PER_CTA");  // tuning overrides
+      const char* er = std::getenv("XR_FLAT_MIN_ROUNDS");
+      // ~1 long unit per resident CTA: each unit's epilogue folds a K-wide
+      // partial row, so long units win (r01 sweep: 256 units 4.7 TB/s, 4096
+      // units 2.5 TB/s on the paper's 2^20 x 2 x 32 int32 gang case)
+      const int64_t want = (eu ? std::max(1, std::atoi(eu)) : 1) * target_ctas;
+      const int64_t min_rounds = er ? std::max(1, std::atoi(er)) : 16;
+      int64_t S = std::max<int64_t>(1, cdiv(want, B));
+      S = std::min<int64_t>(S, std::max<int64_t>(1, nblk / min_rounds));  // >= min_rounds 4 KiB rounds per unit
+      if (chain_capped) S = std::max<int64_t>(S, cdiv(nblk, (int64_t)kChainCap * kUnroll));
+      S = std::max<int64_t>(1, std::min<int64_t>(S, nblk));
+      const int64_t G2 = cdiv(S, kGroupFold);
+      p->kernel = K_COLFLAT;
+      p->vec = vec;
+      p->splits = S;
+      p->units = B * S;
+      p->group = kBlock;
+      if (S > 1) {
+        p->ws_bytes = B * (S + G2) * K * asz;
+        p->tickets = B * (G2 + 1);
+      }
+      ColArgs& c = p->col;
+      c.B = B; c.R = R; c.K = K; c.tiles = 1; c.S = S; c.units = p->units; c.G2 = G2;
+      return;
+    }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
     if (!seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {

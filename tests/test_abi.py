@@ -106,7 +106,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     shape, cd = SHAPE_TABLE[levels]
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
-    assert p["kernel"] in (("col", "coltma") if shape in ("RK", "KRK") else ("seg", "stream", "rows"))
+    assert p["kernel"] in (("col", "coltma", "colflat") if shape in ("RK", "KRK") else ("seg", "stream", "rows"))
 
 
 def test_plan_canonical_cfg2_cfg3_cfg5(xr):
@@ -153,6 +153,10 @@ def test_plan_fp32_chain_cap(xr, case):
         c = p["cdims"]
         work = {"R": c[0], "KR": c[1], "RKR": c[0] * c[2]}[p["shape"]]
         per_acc = work / p["splits"] / (p["group"] * p["vec"] * 4)
+    elif p["kernel"] == "colflat":  # 4 accumulators per thread, one vector per 4 KiB round
+        R = p["cdims"][0] if p["shape"] == "RK" else p["cdims"][1]
+        K = p["cdims"][1] if p["shape"] == "RK" else p["cdims"][2]
+        per_acc = R * K * 4 / 4096 / p["splits"] / 4
     else:  # col: 8 warps x 4 rows in flight; coltma: 4 row phases x 2 accumulators
         R = p["cdims"][0] if p["shape"] == "RK" else p["cdims"][1]
         per_acc = R / p["splits"] / (8 * 4 if p["kernel"] == "col" else 8)

@@ -345,3 +345,19 @@ def test_ring_kernels_stress_repeatable():
         torch.cuda.synchronize()
         for o in outs:
             assert np.array_equal(o.cpu().numpy(), ref), (op, dtype, dims, lv)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [16, 32, 128, 512, 2048, 4096])
+def test_colflat_narrow_rows(dtype, row_bytes, staging):
+    """RK / KRK with power-of-two narrow rows (the flat column kernel): every
+    thread meets a fixed column group; ragged row counts; batches; init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    K = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for dims, lv, op in [((5003, 1, K), "g", "+"), ((3, 1001, K), "w", "max"), ((70001, 1, K), "g", "^" if
+                         dtype.startswith("int") else "*"), ((2, 40000, K), "w", "&&")]:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, sum(dims))
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 3)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
+        if row_bytes <= 512:
+            assert xr.xr_plan_describe(op, dtype, dims, lv, 256)["kernel"] == "colflat"
