@@ -241,6 +241,31 @@ def run_gpu(args):
     for _ in range(max(args.warmup, 3)):
         step()
     torch.cuda.synchronize()
+    exchange = None
+    if comm is not None:
+        # the fused exchange (local reduction + NVLink peer mailboxes in ONE
+        # kernel) must agree with the NCCL path; otherwise fall back to NCCL
+        q = comm.query()
+        exchange = "fused-nvlink-mailbox" if q["fused"] else "nccl"
+        if q["fused"]:
+            step()
+            torch.cuda.synchronize()
+            fused_val = out.clone()
+            comm.set_fused(False)
+            step()
+            torch.cuda.synchronize()
+            nccl_val = out.clone()
+            ok = bool(torch.equal(fused_val, nccl_val)) if dtype != "fp32" else \
+                bool(torch.allclose(fused_val.double(), nccl_val.double(), rtol=1e-5))
+            flag = torch.tensor([1 if (ok and comm.query()["status"] == 0) else 0], device="cuda")
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+            if int(flag.item()) == 1:
+                comm.set_fused(True)
+            else:
+                exchange = "nccl (fused exchange disagreed or timed out; disabled)"
+            for _ in range(3):
+                step()
+            torch.cuda.synchronize()
 
     clocks = ClockSampler(local)
     clocks.start()
@@ -330,7 +355,7 @@ def run_gpu(args):
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": DTYPE_TAG[dtype],
             "data": "synthetic (seeded splitmix64 generator, datagen/)",
-            "config": workload_desc(wl, n, world),
+            "config": dict(workload_desc(wl, n, world), **({"exchange": exchange} if exchange else {})),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,

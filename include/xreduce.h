@@ -297,9 +297,29 @@ int xr_comm_get_unique_id(void* id128);
 int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int device);
 int xr_comm_destroy(xr_comm_t comm);
 
-/* Local xr_reduce on this rank's gang slice + ONE collective on `stream`. */
+/* Fused exchange (default when set up): for whole-nest results (every level
+ * reduced, or the kept ones of extent 1) the last CTA of the local reduction
+ * writes its value into every peer's mailbox over NVLink (CUDA IPC, handles
+ * all-gathered by xr_comm_init), publishes an epoch flag, waits for all ranks
+ * and combines the values in rank order -- ONE kernel, no NCCL launch, the same
+ * bits on every rank.  Set up at xr_comm_init if every peer can be mapped;
+ * otherwise (or when disabled) the NCCL collectives below are used.  The wait
+ * is bounded: a rank that never arrives sets the status read by
+ * xr_comm_query instead of hanging the GPU. */
+int xr_comm_set_fused(xr_comm_t comm, int enable);
+int xr_comm_query(xr_comm_t comm, int* fused, int* status);
+
+/* Local xr_reduce on this rank's gang slice + ONE collective on `stream`
+ * (or the fused exchange above). */
 int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
                       const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream);
+
+/* Single-device simulation of the fused exchange: nranks concurrent kernels on
+ * separate streams, each reducing shards[r] into outs[r] (1 element) with its
+ * own mailbox -- the real publish / spin / combine protocol.  Synchronous.
+ * XR_ERR_NCCL if a rank never arrived. */
+int xr_reduce_fused_sim(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                        const void* const* shards, int nranks, void* const* outs);
 
 /* Single-device simulation of the sharded protocol (testing without NCCL):
  * shards[r] (DEVICE) holds rank r's slice; runs the nranks local reductions

@@ -96,6 +96,9 @@ _SIGS = {
     "xr_comm_destroy": (_c, [_vp]),
     "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
+    "xr_reduce_fused_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, ctypes.POINTER(_vp)]),
+    "xr_comm_set_fused": (_c, [_vp, _c]),
+    "xr_comm_query": (_c, [_vp, ctypes.POINTER(_c), ctypes.POINTER(_c)]),
     "xr_transform_reduce": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_paper": (_c, [_c, _c, _i64p, _u, _vp, _vp, _c, _c, _c, _vp]),
     "xr_reduce_multi": (_c, [_c, ctypes.POINTER(Var), _i64p, _u, _vp]),
@@ -185,6 +188,13 @@ def xr_shutdown() -> int:
 
 def xr_launch_count() -> int:
     return int(_lib.xr_launch_count())
+
+
+def xr_reduce_fused_sim(op, dtype, local_dims, level_mask, shard_ptrs, out_ptrs) -> int:
+    a = (_vp * len(shard_ptrs))(*shard_ptrs)
+    o = (_vp * len(out_ptrs))(*out_ptrs)
+    return _lib.xr_reduce_fused_sim(_op(op), _dt(dtype), _dims(local_dims), mask_of(level_mask), a,
+                                    len(shard_ptrs), o)
 
 
 def xr_heat_step(nj, ni, t1_ptr, t2_ptr, residual_ptr, stream: int = 0) -> int:
@@ -304,6 +314,14 @@ class Comm:
     @property
     def handle(self):
         return self._h
+
+    def set_fused(self, enable: bool) -> int:
+        return _lib.xr_comm_set_fused(self._h, 1 if enable else 0)
+
+    def query(self):
+        f, st = ctypes.c_int(0), ctypes.c_int(0)
+        _check(_lib.xr_comm_query(self._h, ctypes.byref(f), ctypes.byref(st)), "xr_comm_query")
+        return {"fused": bool(f.value), "status": st.value}
 
     def close(self):
         if self._h:

@@ -119,9 +119,11 @@ static cudaError_t gather_dtype(int op, int dtype, const void* g, int nranks, in
   }
 }
 
-// Validated launch (caller holds no lock).
+// Validated launch (caller holds no lock).  exch != nullptr: fused cross-GPU
+// exchange of a whole-nest result (returns XR_ERR_UNSUPPORTED if the plan has
+// no single-output CTA-wide tier to host it).
 static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, const void* in,
-                         void* out, cudaStream_t stream) {
+                         void* out, cudaStream_t stream, const ExchArgs* exch = nullptr) {
   int64_t total = 0, count = 0;
   int st = validate(op, dtype, dims, mask, &total, &count);
   if (st) return st;
@@ -138,6 +140,13 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   Plan p;
   make_plan(op, dtype, dims, mask & 7u, (uint64_t)(uintptr_t)in, sms, &p);
   if (p.kernel == K_NONE) return XR_OK;
+  if (exch) {
+    const bool ok = p.out_count == 1 &&
+                    (p.kernel == K_STREAM || (p.kernel == K_SEG && p.group == kBlock));
+    if (!ok) return XR_ERR_UNSUPPORTED;
+    p.seg.use_exch = 1;
+    p.seg.exch = *exch;
+  }
   Workspace& w = g_ws[{dev, (uintptr_t)stream}];
   // tickets are followed by the two 64-bit scheduler counters (8-B aligned)
   const int64_t tick_words = (p.tickets + 1) & ~int64_t(1);
@@ -397,13 +406,66 @@ int xr_reduce_sharded_sim(int op, int dtype, const int64_t local_dims[3], unsign
   return st;
 }
 
+int xr_reduce_fused_sim(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                        const void* const* shards, int nranks, void* const* outs) {
+  int64_t total = 0, count = 0;
+  int st = validate(op, dtype, local_dims, level_mask, &total, &count);
+  if (st) return st;
+  if (nranks < 1 || nranks > kMaxRanks || !shards || !outs || !(level_mask & XR_GANG) || count != 1)
+    return XR_ERR_INVALID;
+  const size_t mb_bytes = kMailboxWords * sizeof(unsigned long long);
+  unsigned long long* mb = nullptr;
+  int* status = nullptr;
+  if (cudaMalloc(&mb, mb_bytes * nranks) != cudaSuccess || cudaMalloc(&status, sizeof(int)) != cudaSuccess) {
+    cudaGetLastError();
+    return XR_ERR_NOMEM;
+  }
+  cudaMemset(mb, 0, mb_bytes * nranks);
+  cudaMemset(status, 0, sizeof(int));
+  std::vector<cudaStream_t> ss(nranks);
+  for (int r = 0; r < nranks; ++r) cudaStreamCreateWithFlags(&ss[r], cudaStreamNonBlocking);
+  // warm-up per stream (workspace growth, lazy module loading): both may
+  // synchronise the device, which must not happen while a rank's last CTA
+  // spins waiting for the others
+  unsigned long long saved = 0;  // rank 0's initial value survives the warm-up
+  cudaMemcpy(&saved, outs[0], dtype_size(dtype), cudaMemcpyDeviceToHost);
+  for (int r = 0; r < nranks && !st; ++r)
+    st = reduce_device(op, dtype, local_dims, level_mask & 7u, shards[r], outs[r], ss[r]);
+  cudaDeviceSynchronize();
+  cudaMemcpy(outs[0], &saved, dtype_size(dtype), cudaMemcpyHostToDevice);
+  // every "rank" is a concurrent kernel on its own stream; the last CTA of
+  // each spins on its mailbox until all the others published (real protocol)
+  for (int r = 0; r < nranks && !st; ++r) {
+    ExchArgs x{};
+    x.mine = mb + (size_t)r * kMailboxWords;
+    for (int p = 0; p < nranks; ++p) x.peers[p] = mb + (size_t)p * kMailboxWords;
+    x.nranks = nranks;
+    x.rank = r;
+    x.epoch = 1;
+    x.status = status;
+    xr_shard_info info;
+    xr_shard_plan(op, dtype, local_dims, level_mask, nranks, r, &info);
+    const unsigned m = (level_mask & 7u) | (info.local_init_from_out ? XR_INIT_FROM_OUT : 0u);
+    st = reduce_device(op, dtype, local_dims, m, shards[r], outs[r], ss[r], &x);
+  }
+  cudaDeviceSynchronize();
+  int h_status = 0;
+  cudaMemcpy(&h_status, status, sizeof(int), cudaMemcpyDeviceToHost);
+  for (int r = 0; r < nranks; ++r) cudaStreamDestroy(ss[r]);
+  cudaFree(mb);
+  cudaFree(status);
+  if (cudaGetLastError() != cudaSuccess) return XR_ERR_CUDA;
+  if (!st && h_status) st = XR_ERR_NCCL;  // a rank never arrived
+  return st;
+}
+
 }  // extern "C"
 
 namespace xr {
 // used by xr_comm.cpp
 int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask, const void* in, void* out,
-                          cudaStream_t s) {
-  return reduce_device(op, dtype, dims, mask, in, out, s);
+                          cudaStream_t s, const ExchArgs* exch) {
+  return reduce_device(op, dtype, dims, mask, in, out, s, exch);
 }
 cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s) {
   return gather_dtype(op, dtype, g, nranks, n, out, s);

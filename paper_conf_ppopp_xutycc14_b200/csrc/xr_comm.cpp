@@ -8,6 +8,7 @@
 // equivalent for gang partial reduction, @25998-26464), then ONE collective
 // over NVLink/NVSwitch combines them (xr_shard_plan decides which).
 #include <cstring>
+#include <vector>
 #include <nccl.h>
 
 #include "../../include/xreduce.h"
@@ -15,19 +16,66 @@
 
 namespace xr {
 int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask, const void* in, void* out,
-                          cudaStream_t s);
+                          cudaStream_t s, const ExchArgs* exch = nullptr);
 cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
 int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* je);
 int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
                    double* residual, cudaStream_t s);
 }  // namespace xr
 
+using xr::kMaxRanks;
+using xr::kMailboxWords;
+using xr::ExchArgs;
+
 struct xr_comm_s {
   ncclComm_t nccl = nullptr;
   int nranks = 0, rank = 0, device = 0;
   void* scratch = nullptr;  // allgather buffers for & | ^
   size_t scratch_bytes = 0;
+  // fused exchange (peer mailboxes over NVLink via CUDA IPC)
+  bool fused = false;                         // set up and enabled
+  unsigned long long* mailbox = nullptr;      // mine
+  unsigned long long* peers[kMaxRanks] = {};  // every rank's mailbox, mapped into this process
+  int* status = nullptr;
+  unsigned long long epoch = 0;
 };
+
+// Allocate this rank's mailbox, all-gather the CUDA IPC handles with NCCL and
+// map every peer's mailbox.  Any failure leaves the communicator on NCCL.
+static void setup_fused(xr_comm_s* c) {
+  if (c->nranks > kMaxRanks) return;
+  const size_t bytes = kMailboxWords * sizeof(unsigned long long);
+  if (cudaMalloc(&c->mailbox, bytes) != cudaSuccess || cudaMalloc(&c->status, sizeof(int)) != cudaSuccess) {
+    cudaGetLastError();
+    return;
+  }
+  cudaMemset(c->mailbox, 0, bytes);
+  cudaMemset(c->status, 0, sizeof(int));
+  c->peers[c->rank] = c->mailbox;
+  if (c->nranks > 1) {
+    cudaIpcMemHandle_t h;
+    if (cudaIpcGetMemHandle(&h, c->mailbox) != cudaSuccess) { cudaGetLastError(); return; }
+    char* d = nullptr;
+    if (cudaMalloc(&d, (size_t)(c->nranks + 1) * sizeof h) != cudaSuccess) { cudaGetLastError(); return; }
+    cudaMemcpy(d, &h, sizeof h, cudaMemcpyHostToDevice);
+    const bool ok = ncclAllGather(d, d + sizeof h, sizeof h, ncclChar, c->nccl, 0) == ncclSuccess;
+    std::vector<cudaIpcMemHandle_t> all(c->nranks);
+    cudaMemcpy(all.data(), d + sizeof h, c->nranks * sizeof h, cudaMemcpyDeviceToHost);  // syncs stream 0
+    cudaFree(d);
+    if (!ok) return;
+    for (int p = 0; p < c->nranks; ++p) {
+      if (p == c->rank) continue;
+      void* ptr = nullptr;
+      if (cudaIpcOpenMemHandle(&ptr, all[p], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+      }
+      c->peers[p] = static_cast<unsigned long long*>(ptr);
+    }
+  }
+  cudaDeviceSynchronize();
+  c->fused = cudaGetLastError() == cudaSuccess;
+}
 
 using namespace xr;
 
@@ -63,13 +111,42 @@ int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int d
     delete c;
     return XR_ERR_NCCL;
   }
+  setup_fused(c);
   *comm = c;
+  return XR_OK;
+}
+
+int xr_comm_set_fused(xr_comm_t comm, int enable) {
+  if (!comm) return XR_ERR_INVALID;
+  if (enable && !comm->mailbox) return XR_ERR_UNSUPPORTED;
+  if (enable) {  // re-check that every peer is mapped
+    for (int p = 0; p < comm->nranks; ++p)
+      if (!comm->peers[p]) return XR_ERR_UNSUPPORTED;
+  }
+  comm->fused = enable != 0;
+  return XR_OK;
+}
+
+int xr_comm_query(xr_comm_t comm, int* fused, int* status) {
+  if (!comm) return XR_ERR_INVALID;
+  if (fused) *fused = comm->fused ? 1 : 0;
+  if (status) {
+    *status = 0;
+    if (comm->status && cudaMemcpy(status, comm->status, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess) {
+      cudaGetLastError();
+      return XR_ERR_CUDA;
+    }
+  }
   return XR_OK;
 }
 
 int xr_comm_destroy(xr_comm_t comm) {
   if (!comm) return XR_ERR_INVALID;
   int st = XR_OK;
+  for (int p = 0; p < comm->nranks && p < kMaxRanks; ++p)
+    if (p != comm->rank && comm->peers[p]) cudaIpcCloseMemHandle(comm->peers[p]);
+  if (comm->mailbox) cudaFree(comm->mailbox);
+  if (comm->status) cudaFree(comm->status);
   if (comm->scratch) cudaFree(comm->scratch);
   if (comm->nccl && ncclCommDestroy(comm->nccl) != ncclSuccess) st = XR_ERR_NCCL;
   delete comm;
@@ -112,6 +189,19 @@ int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned l
     return XR_OK;
   }
 
+  if (comm->fused && (level_mask & XR_GANG) && info.global_count == 1) {
+    // one kernel: local reduction + peer-mailbox exchange over NVLink
+    ExchArgs x{};
+    x.mine = comm->mailbox;
+    for (int p = 0; p < comm->nranks; ++p) x.peers[p] = comm->peers[p];
+    x.nranks = comm->nranks;
+    x.rank = comm->rank;
+    x.epoch = ++comm->epoch;
+    x.status = comm->status;
+    st = reduce_device_checked(op, dtype, local_dims, base, in_local, mine, s, &x);
+    if (st != XR_ERR_UNSUPPORTED) return st;
+    --comm->epoch;  // this plan cannot host the exchange: NCCL below
+  }
   if ((st = reduce_device_checked(op, dtype, local_dims, base, in_local, mine, s))) return st;
   if (comm->nranks == 1) return XR_OK;
   if (info.collective == XR_COLL_ALLREDUCE) {

@@ -19,6 +19,22 @@ constexpr int kStages = 4;          // bulk-copy ring depth (stream kernel)
 constexpr int64_t kSmallBytes = int64_t(16) << 20;  // below: register kernels (latency bound)
 constexpr int kStageBytes = 16384;  // bytes per stage
 
+// Fused cross-GPU exchange of a whole-nest result (stretch): the
+// last CTA writes its rank's value into every peer's mailbox over NVLink
+// (CUDA IPC peer pointers), publishes an epoch flag, waits for all ranks and
+// combines the nranks values in rank order -- no separate collective launch.
+// Mailbox (uint64 words): [2 parities][kMaxRanks] value slots, then
+// [kMaxRanks] epoch flags.
+constexpr int kMaxRanks = 8;
+constexpr int kMailboxWords = 3 * kMaxRanks;
+struct ExchArgs {
+  unsigned long long* mine;                 // this rank's mailbox
+  unsigned long long* peers[kMaxRanks];     // every rank's mailbox (peers[rank] == mine)
+  int nranks, rank;
+  unsigned long long epoch;                 // > 0, increments per call
+  int* status;                              // set to 1 if a peer never arrived (bounded spin)
+};
+
 // Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]
 // -- covers R (O=1, C=1), KR (C=1) and RKR (C = outer reduced extent).
 struct SegArgs {
@@ -31,6 +47,8 @@ struct SegArgs {
   int64_t Sr, Sc;      // splits over rows and over columns; S = Sr*Sc per output
   int64_t units;       // O * S
   int init_from_out;
+  int use_exch;          // 1: fused exchange of the O == 1 result (exch below)
+  ExchArgs exch;
 };
 
 // Columns ("col"): out[b][c] = (+)_{r<R} in[b][r][c]  -- covers RK (B=1) and KRK.

@@ -114,6 +114,43 @@ __device__ __forceinline__ typename Op<OP, T>::Acc seg_unit(const SegArgs& a, in
   return fold_acc<OP, T, U, VEC>(acc);
 }
 
+// Fused exchange (one thread): publish `mine` to every rank's mailbox, wait for
+// all ranks (bounded), then out[0] = combine of the nranks values in rank
+// order -- identical bits on every rank.  `mine` already carries this rank's
+// share of the initial value (rank 0 only, xr_shard_plan).
+template <int OP, typename T>
+__device__ __noinline__ void peer_exchange(const ExchArgs& ex, T* out, T mine) {
+  const ExchArgs* x = &ex;
+  using O = Op<OP, T>;
+  unsigned long long bits = 0ull;
+  memcpy(&bits, &mine, sizeof(T));
+  const int par = (int)(x->epoch & 1ull);
+  for (int p = 0; p < x->nranks; ++p) x->peers[p][par * kMaxRanks + x->rank] = bits;  // NVLink stores
+  // each flag store is a release at system scope: it orders this thread's
+  // slot stores above before the flag becomes visible to the peer
+  for (int p = 0; p < x->nranks; ++p) {
+    unsigned long long* f = x->peers[p] + 2 * kMaxRanks + x->rank;
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(x->epoch) : "memory");
+  }
+  typename O::Acc acc = O::identity();
+  for (int q = 0; q < x->nranks; ++q) {
+    const unsigned long long* f = x->mine + 2 * kMaxRanks + q;
+    unsigned long long e = 0ull;
+    for (long long spin = 0; spin < (1ll << 26); ++spin) {
+      asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(e) : "l"(f) : "memory");
+      if (e >= x->epoch) break;
+      __nanosleep(64);
+    }
+    if (e < x->epoch) *x->status = 1;  // a peer never arrived: report instead of hanging
+    unsigned long long v;
+    asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(x->mine + par * kMaxRanks + q) : "memory");
+    T tv;
+    memcpy(&tv, &v, sizeof(T));
+    acc = O::combine(acc, O::lift(tv));
+  }
+  out[0] = O::finish(acc);
+}
+
 // a5: out[o] = init (+) R, init = identity or the prior out[o] (@21488-21990).
 template <int OP, typename T>
 __device__ __forceinline__ T merge_init(typename Op<OP, T>::Acc v, const T* out, int64_t o,
@@ -169,7 +206,11 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
       Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
       v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
       if (S == 1) {
-        if (threadIdx.x == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+        if (threadIdx.x == 0) {
+          const T r = merge_init<OP, T>(v, out, o, a.init_from_out);
+          if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
+          else out[o] = r;
+        }
       } else {  // a4: gang tier, last CTA of output o combines its S partials
         if (threadIdx.x == 0) {
           partials[u] = v;
@@ -183,8 +224,10 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
           Acc w = fold_partials<OP, T>(partials + o * S, S, threadIdx.x, BLOCK);
           w = block_reduce<OP, T, BLOCK>(w, smem);
           if (threadIdx.x == 0) {
-            out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+            const T r = merge_init<OP, T>(w, out, o, a.init_from_out);
             a.tickets[o] = 0u;  // self-resetting for the next launch
+            if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
+            else out[o] = r;
           }
         }
       }
@@ -413,8 +456,10 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
       Acc w = fold_partials<OP, T>(partials, S, ct, kConsThreads);
       w = cons_reduce<OP, T>(w, smem, cw, lane);
       if (ct == 0) {
-        out[0] = merge_init<OP, T>(w, out, 0, a.init_from_out);
+        const T r = merge_init<OP, T>(w, out, 0, a.init_from_out);
         a.tickets[0] = 0u;
+        if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
+        else out[0] = r;
       }
     }
   }

@@ -65,3 +65,22 @@ def test_heat_sharded_one_rank(comm):
     assert res.cpu().tolist() == ref_res.tolist()
     fin = (t1 if iters % 2 == 0 else t2).cpu().numpy().reshape(nj + 2, ni)[1:nj + 1]
     assert np.array_equal(fin.view(np.uint64), ref_T.reshape(nj, ni).view(np.uint64))
+
+
+def test_fused_exchange_one_rank(comm):
+    """The real communicator with the fused exchange (1 rank: the mailbox is
+    local) and with it disabled (NCCL): both equal the oracle."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    assert comm.query()["fused"]
+    n = (1 << 22) + 7
+    x = recipes.make("ints", (n, 1, 1), 7, "int64", 5)
+    ref = oracle.reduce("+", "int64", (n, 1, 1), "gwv", x)
+    xd = torch.from_numpy(x).cuda()
+    for fused in (True, False, True):
+        assert comm.set_fused(fused) == 0
+        for _ in range(3):  # epochs advance, parity slots alternate
+            out = xr.reduce_sharded(xd, comm, "+", "gwv", nest_local=(n, 1, 1))
+            torch.cuda.synchronize()
+            assert out.cpu().numpy()[:1].tolist() == ref.tolist()
+    assert comm.query()["status"] == 0
