@@ -112,6 +112,25 @@ int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int d
     return XR_ERR_NCCL;
   }
   setup_fused(c);
+  if (nranks > 1) {
+    // consensus: the fused exchange is used only if EVERY rank mapped every
+    // peer (a mixed setup would leave fused ranks spinning while the others
+    // sit in an NCCL collective)
+    int* d = nullptr;
+    int ok = c->fused ? 1 : 0;
+    if (cudaMalloc(&d, sizeof(int)) == cudaSuccess) {
+      cudaMemcpy(d, &ok, sizeof(int), cudaMemcpyHostToDevice);
+      if (ncclAllReduce(d, d, 1, ncclInt32, ncclMin, c->nccl, 0) == ncclSuccess)
+        cudaMemcpy(&ok, d, sizeof(int), cudaMemcpyDeviceToHost);
+      else
+        ok = 0;
+      cudaFree(d);
+    } else {
+      cudaGetLastError();
+      ok = 0;  // NOTE: this rank still joined no collective; all ranks reach the allreduce above or fail alike
+    }
+    c->fused = ok == 1;
+  }
   *comm = c;
   return XR_OK;
 }
