@@ -191,7 +191,8 @@ typedef struct {
   int kernel;           /* 0 none, 1 fill, 2 ident, 3 seg, 4 col, 5 stream,
                            6 coltma (TMA tensor-map column kernel),
                            7 rows (bulk-streamed short contiguous rows),
-                           8 colflat (narrow-row column reduction)           */
+                           8 colflat (narrow-row column reduction),
+                           9 rkr (bulk-streamed rows folded by middle index) */
   int64_t cdims[3];     /* canonical extents (shape-dependent, rest 0)       */
   int64_t out_count;
   int group;            /* seg: lanes per group (8, 32 or the CTA size)      */

@@ -161,6 +161,8 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   p.col.in = in; p.col.out = out; p.col.partials = w.partials; p.col.tickets = w.tickets;
   p.col.init_from_out = ifo;
   p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
+  p.rkr.in = in; p.rkr.out = out; p.rkr.partials = w.partials; p.rkr.tickets = w.tickets;
+  p.rkr.sched = sched; p.rkr.init_from_out = ifo;
   if (p.kernel == K_COLTMA && !make_col_tmap(&p.tmap, dtype, in, p.col.B, p.col.R, p.col.K)) {
     // no tensor-map support: re-plan without TMA (same workspace bound or smaller)
     return XR_ERR_CUDA;
@@ -244,7 +246,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   info->units = p.units;
   info->block = p.block;
   int64_t ctas = p.units;
-  if (p.kernel == K_STREAM || p.kernel == K_COLTMA || p.kernel == K_ROWS) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
+  if (p.kernel == K_STREAM || p.kernel == K_COLTMA || p.kernel == K_ROWS || p.kernel == K_RKR) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);

@@ -13,7 +13,7 @@ constexpr int kChainCap = 4096; // max sequential fp32 '+' chain per accumulator
 constexpr int kTargetCtasPerSm = 8;  // 2048 threads/SM at 256 threads/CTA
 constexpr int kUnitsPerCta = 8;      // dynamic units per resident CTA (tail balance)
 
-enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6, K_ROWS = 7, K_COLFLAT = 8 };
+enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6, K_ROWS = 7, K_COLFLAT = 8, K_RKR = 9 };
 
 constexpr int kStages = 4;          // bulk-copy ring depth (stream kernel)
 constexpr int64_t kSmallBytes = int64_t(16) << 20;  // below: register kernels (latency bound)
@@ -75,6 +75,18 @@ struct EltArgs {
   int init_from_out;
 };
 
+// RKR rows kernel (xr_kernels.cuh rkr_kernel)
+struct RkrArgs {
+  const void* in;
+  void* out;
+  void* partials;          // [S][K] then [G2][K]
+  unsigned* tickets;       // [G2] group tickets, then 1 top ticket
+  unsigned long long* sched;
+  int64_t K, L, NR;        // outputs, row length, rows = R1*K
+  int64_t S, G2;           // units, groups
+  int init_from_out;
+};
+
 struct Plan {
   int shape = 0;        // xr_shape
   int kernel = K_NONE;
@@ -92,6 +104,7 @@ struct Plan {
   SegArgs seg{};
   ColArgs col{};
   CUtensorMap tmap{};   // K_COLTMA: 3-D map over (K, R, B), built at launch
+  RkrArgs rkr{};
   EltArgs elt{};
 };
 

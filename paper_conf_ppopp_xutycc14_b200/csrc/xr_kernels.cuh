@@ -745,6 +745,182 @@ __global__ void __launch_bounds__(kBlock) colflat_kernel(ColArgs a) {
   }
 }
 
+// ------------------------------------------------------------- RKR rows kernel
+// RKR (reduce outer k and inner i, keep the middle j) with short rows
+// (row_bytes = L*size a power of two in [512 B, 2 KiB], 16-B aligned): the
+// rows (k, j) are contiguous in memory and row r feeds output j = r mod K, so
+// the whole nest is streamed like the rows kernel (producer warp, bulk copies
+// of 16 KiB stages); each consumer warp reduces its rows (a2) and lane 0
+// folds the result into a shared per-output array acc[K] (a3) -- rows in
+// flight never share an output because K >= 32 >= rows per stage x stages.
+// A unit (a block of whole stages) leaves a K-wide partial row; the gang tier
+// is two-level (unit partials -> groups of kGroupFold -> outputs).
+
+template <int OP, typename T, int NS>
+__global__ void __launch_bounds__(kWsBlock) rkr_kernel(RkrArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int STAGE = kStageBytes;
+  constexpr int RING = 8;
+  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE, then acc[K]
+  __shared__ __align__(8) uint64_t full[NS];
+  __shared__ __align__(8) uint64_t empty[NS];
+  __shared__ long long s_units[RING];
+  __shared__ int s_last;
+  Acc* acc = reinterpret_cast<Acc*>(stage_mem + NS * STAGE);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  T* out = static_cast<T*>(a.out);
+  const int64_t row_bytes = a.L * (int64_t)sizeof(T);
+  const int rshift = __ffsll(row_bytes) - 1;
+  const int rps = (int)(STAGE >> rshift);
+  const int64_t nst = (a.NR + rps - 1) / rps;
+
+  if (tid == 0) {
+#pragma unroll
+    for (int k = 0; k < NS; ++k) {
+      mbar_init(&full[k], 1);
+      mbar_init(&empty[k], kConsWarps);
+    }
+    fence_mbar_init();
+  }
+  __syncthreads();
+
+  if (warp == 0) {  // ---------------- producer warp
+    if (lane == 0) {
+      int64_t g = 0;
+      int seq = 0;
+      long long u = (long long)atomicAdd(a.sched, 1ull);
+      while (true) {
+        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const int slot0 = (int)(g % NS);
+        s_units[seq & (RING - 1)] = u < a.S ? u : -1;
+        ++seq;
+        if (u >= a.S) {
+          if (g >= NS) mbar_wait(&empty[slot0], (unsigned)(((g / NS) - 1) & 1));
+          mbar_arrive(&full[slot0]);
+          break;
+        }
+        const int64_t st0 = split_lo(nst, a.S, u), st1 = split_lo(nst, a.S, u + 1);
+        for (int64_t st = st0; st < st1; ++st, ++g) {
+          const int slot = (int)(g % NS);
+          if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
+          const int64_t row0 = st * rps;
+          const unsigned nb = (unsigned)(min((int64_t)rps, a.NR - row0) << rshift);
+          mbar_expect_tx(&full[slot], nb);
+          bulk_g2s(stage_mem + slot * STAGE, static_cast<const char*>(a.in) + (row0 << rshift), nb, &full[slot]);
+        }
+        u = nu;
+      }
+      sched_exit(a.sched);
+    }
+    return;
+  }
+
+  // ---------------- consumer warps
+  const int ct = tid - 32, cw = warp - 1;
+  Acc* partials = static_cast<Acc*>(a.partials);
+  Acc* P2 = partials + a.S * a.K;
+  int seq = 0;
+  int64_t g = 0;
+  // fold rows [0, n) of a [n][K] partial block into column c (all consumers)
+  auto fold_col = [&](const Acc* src, int64_t n, int64_t c) {
+    Acc z = O::identity();
+    int64_t r = 0;
+    for (; r + 3 < n; r += 4) {
+      Acc y[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) y[k] = ld_partial(src + (r + k) * a.K + c);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) z = O::combine(z, y[k]);
+    }
+    for (; r < n; ++r) z = O::combine(z, ld_partial(src + r * a.K + c));
+    return z;
+  };
+  while (true) {
+    mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
+    const long long u = s_units[seq & (RING - 1)];
+    if (u < 0) break;
+    for (int64_t c = ct; c < a.K; c += kConsThreads) acc[c] = O::identity();
+    cons_sync();
+    const int64_t st0 = split_lo(nst, a.S, u), st1 = split_lo(nst, a.S, u + 1);
+    for (int64_t st = st0; st < st1; ++st, ++g) {
+      const int slot = (int)(g % NS);
+      if (st > st0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+      const int64_t row0 = st * rps;
+      const int nrows = (int)min((int64_t)rps, a.NR - row0);
+      const unsigned char* sm = stage_mem + slot * STAGE;
+      const int rpw = rps / kConsWarps;
+      const int vpl = (int)(row_bytes >> 9);
+      Acc v[4];
+#pragma unroll
+      for (int rr = 0; rr < 4; ++rr) {
+        v[rr] = O::identity();
+        const int r = cw * rpw + rr;
+        if (rr < rpw && r < nrows) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            if (k < vpl) {
+              const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + (k * 32 + lane) * 16);
+#pragma unroll
+              for (int q = 0; q < VEC; ++q) v[rr] = O::combine(v[rr], O::lift(unpack<T>(x, q)));
+            }
+          }
+        }
+      }
+      fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);
+#pragma unroll
+      for (int rr = 0; rr < 4; ++rr) {
+        if (rr < rpw) {
+          const Acc w = group_reduce<OP, T, 32>(v[rr]);
+          const int r = cw * rpw + rr;
+          if (lane == 0 && r < nrows) {
+            const int64_t j = (row0 + r) % a.K;
+            acc[j] = O::combine(acc[j], w);
+          }
+        }
+      }
+    }
+    cons_sync();  // acc[] complete for this unit
+    // a4, two levels: unit partial row -> group -> outputs
+    for (int64_t c = ct; c < a.K; c += kConsThreads) partials[u * a.K + c] = acc[c];
+    const int64_t gi = u / kGroupFold, g0 = gi * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
+    cons_sync();
+    if (ct == 0) {
+      __threadfence();
+      s_last = (atomicAdd(&a.tickets[gi], 1u) == (unsigned)(gsz - 1));
+    }
+    cons_sync();
+    if (s_last) {
+      __threadfence();
+      if (a.G2 == 1) {
+        for (int64_t c = ct; c < a.K; c += kConsThreads)
+          out[c] = merge_init<OP, T>(fold_col(partials + g0 * a.K, gsz, c), out, c, a.init_from_out);
+        if (ct == 0) a.tickets[gi] = 0u;
+      } else {
+        for (int64_t c = ct; c < a.K; c += kConsThreads) P2[gi * a.K + c] = fold_col(partials + g0 * a.K, gsz, c);
+        cons_sync();
+        if (ct == 0) {
+          a.tickets[gi] = 0u;
+          __threadfence();
+          s_last = (atomicAdd(&a.tickets[a.G2], 1u) == (unsigned)(a.G2 - 1));
+        }
+        cons_sync();
+        if (s_last) {
+          __threadfence();
+          for (int64_t c = ct; c < a.K; c += kConsThreads)
+            out[c] = merge_init<OP, T>(fold_col(P2, a.G2, c), out, c, a.init_from_out);
+          if (ct == 0) a.tickets[a.G2] = 0u;
+        }
+      }
+    }
+    cons_sync();
+    ++seq;
+  }
+}
+
 // ------------------------------------------------------------- col kernel
 // Lanes own VEC contiguous kept columns (a 32*VEC-column tile per warp row);
 // the CTA's warps stride over the reduced rows of a row chunk; the worker tier
@@ -1160,6 +1336,22 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
         return n;
       }();
       kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsBlock, dyn, s>>>(p.seg);
+      break;
+    }
+    case K_RKR: {
+      auto kern = rkr_kernel<OP, T, kStages>;
+      const int dyn = kStages * kStageBytes + (int)(p.rkr.K * sizeof(typename Op<OP, T>::Acc));
+      static int occ = [&] {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kStages * kStageBytes + 16384);
+        int n = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, kStages * kStageBytes + 16384) !=
+                cudaSuccess || n < 1)
+          n = 1;
+        return n;
+      }();
+      int64_t grid = grid_for(p.units, num_sms, occ);
+      if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
+      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.rkr);
       break;
     }
     case K_ROWS: {

@@ -228,6 +228,34 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   else { O = run_n[1]; C = run_n[0]; L = run_n[2]; rowStride = O * L; oStride = L; p->shape = XR_SHAPE_RKR; }
 
   const int64_t row_bytes = L * size;
+  // RKR with short rows: stream all rows, fold by output in shared memory.
+  // OPT-IN (XR_RKR=1): measured r01 on 512^3 int32/fp32 GV at 0.60 of peak vs
+  // 0.82 for the seg path -- its K-wide partial-row folds are latency bound.
+  if (!seg_only && !seg_only_small && nr == 3 && std::getenv("XR_RKR") != nullptr &&
+      row_bytes >= 512 && row_bytes <= 2048 &&
+      (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= 32 && O * asz <= 16384 &&
+      std::getenv("XR_NO_BULK") == nullptr) {
+    const int64_t rps = kStageBytes / row_bytes;
+    const int64_t NR = C * O;
+    const int64_t nst = cdiv(NR, rps);
+    const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;
+    const int64_t k = 2;  // equal units per CTA
+    int64_t S = std::max<int64_t>(1, std::min<int64_t>(nst / kStages, k * cap));
+    if (chain_capped) S = std::max<int64_t>(S, cdiv(NR, (int64_t)kChainCap * 8));
+    const int64_t G2 = cdiv(S, kGroupFold);
+    p->kernel = K_RKR;
+    p->group = 32;
+    p->vec = vec;
+    p->splits = S;
+    p->units = S;
+    p->sched = true;
+    p->grid_hint = std::min<int64_t>(cap, cdiv(S, k));
+    p->ws_bytes = (S + G2) * O * asz;
+    p->tickets = G2 + 1;
+    RkrArgs& r = p->rkr;
+    r.K = O; r.L = L; r.NR = NR; r.S = S; r.G2 = G2;
+    return;
+  }
   // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
   // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
   if (!seg_only && !seg_only_small && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 &&

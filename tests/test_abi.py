@@ -106,7 +106,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     shape, cd = SHAPE_TABLE[levels]
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
-    assert p["kernel"] in (("col", "coltma", "colflat") if shape in ("RK", "KRK") else ("seg", "stream", "rows"))
+    assert p["kernel"] in (("col", "coltma", "colflat") if shape in ("RK", "KRK") else ("seg", "stream", "rows", "rkr"))
 
 
 def test_plan_canonical_cfg2_cfg3_cfg5(xr):
@@ -147,7 +147,9 @@ def test_plan_fp32_chain_cap(xr, case):
     """fp32 '+' keeps every accumulator's sequential chain <= 4096 (C9)."""
     _, dims, lv = case
     p = xr.xr_plan_describe("+", "fp32", dims, lv, 256)
-    if p["kernel"] == "rows":
+    if p["kernel"] == "rkr":
+        per_acc = p["cdims"][0] * p["cdims"][2] / p["splits"] / 32  # per lane: rows x VEC per unit
+    elif p["kernel"] == "rows":
         per_acc = p["cdims"][1] / (32 * p["vec"])  # one row per warp-wide fold, VEC chains per lane
     elif p["kernel"] in ("seg", "stream"):
         c = p["cdims"]

@@ -361,3 +361,21 @@ def test_colflat_narrow_rows(dtype, row_bytes, staging):
         check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
         if row_bytes <= 512:
             assert xr.xr_plan_describe(op, dtype, dims, lv, 256)["kernel"] == "colflat"
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [512, 1024, 2048])
+def test_rkr_kernel_short_rows(dtype, row_bytes, monkeypatch):
+    """RKR (gang + vector reduced, worker kept) with short rows: the bulk-
+    streamed rows folded by their middle index (forced with XR_SMALL_BYTES=0)."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    monkeypatch.setenv("XR_RKR", "1")  # opt-in kernel (DESIGN.md: slower than seg on 512^3)
+    L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for R1, K, op in [(7, 32, "+"), (33, 100, "max"), (5, 999, "&&"), (300, 40, "*")]:
+        dims = (R1, K, L)
+        x = recipes.make(KIND[op], dims, oracle.mask_of("gv"), dtype, R1 * K)
+        init = recipes.make("ints", (K, 1, 1), 1, dtype, 4)
+        check(op, dtype, dims, "gv", gpu_reduce(op, dtype, dims, "gv", x, init=init), x, init=init)
+        if K * (8 if dtype == "int64" or dtype == "fp64" else 4) <= 16384:
+            assert xr.xr_plan_describe(op, dtype, dims, "gv", 256)["kernel"] == "rkr"
