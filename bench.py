@@ -171,6 +171,22 @@ def oracle_rate(wl, x_sample: np.ndarray, seconds: float):
     return reps * n / el, reps, el
 
 
+def openmp_rate(wl, x_sample: np.ndarray, seconds: float):
+    """The all-cores OpenMP CPU baseline (cpubase/) on the same sample."""
+    import cpubase
+    op, dtype, _, _ = WORKLOADS[wl]
+    n = x_sample.size
+    cpubase.reduce(op, dtype, (n, 1, 1), "gwv", x_sample)  # spin up the thread pool
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        cpubase.reduce(op, dtype, (n, 1, 1), "gwv", x_sample)
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            break
+    return reps * n / el, reps, el, cpubase.num_procs()
+
+
 def run_reference(args):
     rank, world, _ = dist_env()
     if rank != 0:
@@ -342,12 +358,16 @@ def run_gpu(args):
                "api": "xr_reduce_host (C ABI, pinned host input)" if world == 1 else
                       "pinned H2D + xr_reduce_sharded + D2H"}
 
-    cpu = None
+    cpu = cpu_omp = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sample_n = min(n, 1 << 26)
         rate, reps, el = oracle_rate(wl, host.numpy()[:sample_n], args.cpu_seconds)
         cpu = {"value": rate, "unit": "elements/s", "cores": 1, "kind": "oracle",
                "sample": f"{reps} x oracle over the first {sample_n} elements ({el:.1f} s, 1 thread)"}
+        rate, reps, el, cores = openmp_rate(wl, host.numpy()[:sample_n], min(args.cpu_seconds, 3.0))
+        cpu_omp = {"value": rate, "unit": "elements/s", "cores": cores, "kind": "openmp",
+                   "sample": f"{reps} x cpubase/omp.c over the first {sample_n} elements ({el:.1f} s, "
+                             f"{cores} threads)"}
 
     if rank == 0:
         line = {
@@ -367,6 +387,7 @@ def run_gpu(args):
             "gpu_launches": launches,
             "clocks": ck,
             "cpu_baseline": cpu,
+            "cpu_baseline_openmp": cpu_omp,
         }
         print(json.dumps(line), flush=True)
     if comm is not None:
