@@ -5,11 +5,15 @@ Metric: reduced elements/s (and % of B200 HBM peak) at N GPUs vs the CPU oracle.
 Workload (N=1, BASELINE.json configs[1], "cfg2"): 1-D whole-array sum of 2^30
 fp32 elements U[0,1), reduction at gang+worker+vector.  One step = one
 xr_reduce call (the whole hot path: plan, private partials, warp / CTA / last-
-CTA combine, init merge).  N>1 (torchrun): each rank owns its own 2^30-element
-gang slice of a N*2^30 array (weak scaling) and one step = xr_reduce_sharded
-(local kernel + one 4-byte NCCL allreduce over NVLink).
+CTA combine, init merge).  N>1 (torchrun): the same 2^30-element array is
+gang-sharded, rank r owning the contiguous slice r (strong scaling, the
+BASELINE cfg2 reading "1 GPU then sharded 2/4/8 GPUs"), and one step =
+xr_reduce_sharded (local single-pass kernel + one cross-GPU combine: the fused
+NVLink mailbox exchange inside the same kernel, or one NCCL allreduce).
+--scaling weak gives every rank its own 2^30-element slice instead.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
+                  [--scaling strong|weak]
                   [--workload fp32-sum|fp32-max|fp32-min|int64-sum|int64-max|int64-min]
 
 Prints ONE JSON line on rank 0.
@@ -51,7 +55,11 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", default="xreduce", choices=["xreduce", "reference"])
     ap.add_argument("--workload", default="fp32-sum", choices=sorted(WORKLOADS))
-    ap.add_argument("--elements", type=int, default=N_PER_GPU, help="elements per GPU")
+    ap.add_argument("--elements", type=int, default=N_PER_GPU,
+                    help="elements of the whole array (strong scaling) or per GPU (weak)")
+    ap.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                    help="strong (default, BASELINE cfg2: the one 2^30-element array sharded over N GPUs) "
+                         "or weak (2^30 elements per GPU)")
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
@@ -75,11 +83,12 @@ def make_input(wl, n, start, total):
     return recipes.make(kind, (total, 1, 1), 7, dtype, seed, start=start, n=n)
 
 
-def workload_desc(wl, n, world):
+def workload_desc(wl, n, world, scaling="strong"):
     op, dtype, kind, _ = WORKLOADS[wl]
     return {
-        "workload": f"cfg2: 1-D whole-array '{op}' over {n} {dtype} elements per GPU ({kind}), "
-                    f"level_mask gang+worker+vector" + (f", gang-sharded over {world} GPUs + NCCL allreduce"
+        "workload": f"cfg2: 1-D whole-array '{op}' over {n * world} {dtype} elements ({kind}), "
+                    f"level_mask gang+worker+vector" + (f", gang-sharded over {world} GPUs ({n} per GPU, "
+                                                       f"{scaling} scaling) + one cross-GPU combine"
                                                        if world > 1 else ""),
         "nest_dims_per_gpu": [n, 1, 1],
         "level_mask": "gwv",
@@ -192,7 +201,7 @@ def run_reference(args):
     if rank != 0:
         return 0
     wl = args.workload
-    n = args.elements
+    n = args.elements // args.gpus if args.scaling == "strong" else args.elements
     sample_n = min(n, 1 << 24)  # bounded sample per step: the whole run stays within minutes
     x = make_input(wl, sample_n, 0, n)
     per_step = []
@@ -205,9 +214,9 @@ def run_reference(args):
     line = {
         "metric": METRIC, "value": value, "unit": "elements/s", "n_gpus": args.gpus, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": DTYPE_TAG[WORKLOADS[wl][1]],
+        "scaling": args.scaling, "vs_baseline": None, "dtype": DTYPE_TAG[WORKLOADS[wl][1]],
         "data": "synthetic (seeded splitmix64 generator, datagen/)", "impl": "reference",
-        "config": workload_desc(wl, n, args.gpus),
+        "config": workload_desc(wl, n, args.gpus, args.scaling),
         "cpu_baseline": {"value": value, "unit": "elements/s", "cores": 1, "kind": "oracle",
                          "sample": f"first {sample_n} elements of the workload per step (plain C oracle, 1 thread)"},
         "e2e": {"value": value, "unit": "elements/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -233,8 +242,14 @@ def run_gpu(args):
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     wl = args.workload
     op, dtype, kind, esz = WORKLOADS[wl]
-    n = args.elements
-    total = n * world
+    if args.scaling == "strong":  # the whole array is fixed; rank r owns gang slice r
+        total = args.elements
+        if total % world:
+            raise SystemExit(f"--elements {total} is not divisible by {world} GPUs")
+        n = total // world
+    else:
+        n = args.elements
+        total = n * world
     tdt = {"fp32": torch.float32, "int64": torch.int64}[dtype]
 
     # inputs: seeded host generation of this rank's gang slice, pinned, then resident in HBM
@@ -372,10 +387,10 @@ def run_gpu(args):
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": DTYPE_TAG[dtype],
             "data": "synthetic (seeded splitmix64 generator, datagen/)",
-            "config": dict(workload_desc(wl, n, world), **({"exchange": exchange} if exchange else {})),
+            "config": dict(workload_desc(wl, n, world, args.scaling), **({"exchange": exchange} if exchange else {})),
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,

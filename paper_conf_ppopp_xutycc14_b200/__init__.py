@@ -16,7 +16,8 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libxreduce.so")
+# XR_LIB_PATH: load another build of the same library (tools/ A/B variants only)
+LIB_PATH = os.environ.get("XR_LIB_PATH") or os.path.join(_HERE, "libxreduce.so")
 if not os.path.exists(LIB_PATH):
     raise ImportError(
         f"xreduce: {LIB_PATH} is missing -- build the CUDA library first "

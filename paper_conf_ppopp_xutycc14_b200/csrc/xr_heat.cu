@@ -308,9 +308,9 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
     if (lane == 0) {
       int64_t q = 0;  // global row counter (slot = q % kHeatSlots)
       int seq = 0;
-      long long t = (long long)atomicAdd(pa.sched, 1ull);
+      long long t = claim_first();
       while (true) {
-        const long long nt = (long long)atomicAdd(pa.sched, 1ull);
+        const long long nt = claim_next(pa.sched);
         const int slot0 = (int)(q % kHeatSlots);
         s_tiles[seq & (RING - 1)] = t < ntiles ? t : -1;
         ++seq;

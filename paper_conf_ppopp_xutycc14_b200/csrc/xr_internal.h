@@ -75,15 +75,16 @@ struct EltArgs {
   int init_from_out;
 };
 
-// RKR rows kernel (xr_kernels.cuh rkr_kernel)
+// RKR rows kernel (xr_kernels.cuh rkr_kernel): out[j] = (+)_{k<C} (+)_{i<L}
+// in[(k*K + j)*L + i]; units = (j-block of 16 KiB / row_bytes outputs, k split)
 struct RkrArgs {
   const void* in;
   void* out;
-  void* partials;          // [S][K] then [G2][K]
-  unsigned* tickets;       // [G2] group tickets, then 1 top ticket
+  void* partials;          // Acc[K][S] when S > 1
+  unsigned* tickets;       // [K] when S > 1, zero between launches
   unsigned long long* sched;
-  int64_t K, L, NR;        // outputs, row length, rows = R1*K
-  int64_t S, G2;           // units, groups
+  int64_t K, L, C;         // outputs (middle extent), row length, outer reduced extent
+  int64_t S, units;        // k splits per j-block, j-blocks * S
   int init_from_out;
 };
 

@@ -52,6 +52,12 @@ __device__ __forceinline__ void fold_row(const T* __restrict__ row, int64_t n, i
   const int64_t nv = n / VEC;
   const U128* __restrict__ vp = reinterpret_cast<const U128*>(row);
   int64_t v = lane;
+// XR_FOLD_PIPELINE=1: software-pipelined variant (A/B only; more registers,
+// measured no better than the plain loop under __launch_bounds__(256, 4))
+#ifndef XR_FOLD_PIPELINE
+#define XR_FOLD_PIPELINE 0
+#endif
+#if XR_FOLD_PIPELINE == 0
   for (; v + (int64_t)(U - 1) * W < nv; v += (int64_t)U * W) {
     U128 x[U];
 #pragma unroll
@@ -61,6 +67,33 @@ __device__ __forceinline__ void fold_row(const T* __restrict__ row, int64_t n, i
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
   }
+#else
+  if (v + (int64_t)(U - 1) * W < nv) {
+    // software-pipelined: the U loads of round n+1 are issued before round n
+    // is folded, so they have no use inside the iteration and ptxas keeps
+    // them in one batch (it sank unpipelined loads next to their uses,
+    // leaving 2 of 4 in flight: fp64 && || rows at 0.63 of peak, r01)
+    U128 x[U];
+#pragma unroll
+    for (int k = 0; k < U; ++k) x[k] = ld_stream(vp + v + (int64_t)k * W);
+    v += (int64_t)U * W;
+    for (; v + (int64_t)(U - 1) * W < nv; v += (int64_t)U * W) {
+      U128 y[U];
+#pragma unroll
+      for (int k = 0; k < U; ++k) y[k] = ld_stream(vp + v + (int64_t)k * W);
+#pragma unroll
+      for (int k = 0; k < U; ++k)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
+#pragma unroll
+      for (int k = 0; k < U; ++k) x[k] = y[k];
+    }
+#pragma unroll
+    for (int k = 0; k < U; ++k)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
+  }
+#endif
   for (; v < nv; v += W) {
     const U128 x = ld_stream(vp + v);
 #pragma unroll
@@ -180,12 +213,53 @@ __device__ __forceinline__ typename Op<OP, T>::Acc fold_partials(const typename 
   return w;
 }
 
+// Fold a CONTIGUOUS 16-B aligned partial array p[0..n) with 16-B loads (4 or 2
+// accumulators each), 8 in flight per thread: the single-output "whole" mode
+// folds thousands of unit partials after every other CTA has finished, so
+// this tail is latency bound (r01: 9472 partials in 5 rounds of 8 scalar
+// loads per thread -> 2 rounds of 16-B loads).  Fixed order per thread.
+template <int OP, typename T>
+__device__ __forceinline__ typename Op<OP, T>::Acc fold_partials_vec(const typename Op<OP, T>::Acc* p, int64_t n,
+                                                                     int t, int nt) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int PV = 16 / sizeof(Acc);
+  const int64_t nv = n / PV;
+  Acc w = O::identity();
+  int64_t i = t;
+  for (; i + 7 * (int64_t)nt < nv; i += 8 * (int64_t)nt) {
+    U128 y[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k) y[k] = ld_partial16(p + (i + (int64_t)k * nt) * PV);
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+#pragma unroll
+      for (int q = 0; q < PV; ++q) w = O::combine(w, acc_at<Acc>(y[k], q));
+  }
+  for (; i < nv; i += nt) {
+    const U128 y = ld_partial16(p + i * PV);
+#pragma unroll
+    for (int q = 0; q < PV; ++q) w = O::combine(w, acc_at<Acc>(y, q));
+  }
+  for (int64_t e = nv * PV + t; e < n; e += nt) w = O::combine(w, ld_partial(p + e));
+  return w;
+}
+
 // ------------------------------------------------------------- seg kernel
 // Groups of W lanes (8 or 32: inside a warp; W == BLOCK: the whole CTA) each
 // reduce work units; a unit is (output o, split s).  Splits (S > 1) only
 // occur with W >= 32 (plan), so a ticket is always taken by a whole warp/CTA.
 template <int OP, typename T, int W, int BLOCK, int U>
-__global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
+// Minimum resident CTAs in the register kernels' launch bounds (<= 64
+// registers).  It also steers ptxas's scheduling: without it ptxas sank the
+// unrolled 16-B loads of fold_row next to their uses in some instantiations
+// (2 of 4 loads in flight; fp64 && || rows at 0.63 of peak, the paper's
+// 2^20 x 2 x 32 gang case at 64 us instead of 50 us).  r01 A/B, and
+// tests/test_sass.py keeps every fold loop at >= 4 loads in flight.
+#ifndef XR_SEG_MINB
+#define XR_SEG_MINB 4
+#endif
+__global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_constant__ SegArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   __shared__ Acc smem[32];
@@ -196,12 +270,12 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
 
   if constexpr (W == BLOCK) {
     __shared__ long long s_unit[2];
-    if (threadIdx.x == 0) s_unit[0] = (long long)atomicAdd(a.sched, 1ull);
+    if (threadIdx.x == 0) s_unit[0] = claim_first();
     __syncthreads();
     long long u = s_unit[0];
     int par = 1;
     while (u < a.units) {
-      if (threadIdx.x == 0) s_unit[par] = (long long)atomicAdd(a.sched, 1ull);  // next, in flight
+      if (threadIdx.x == 0) s_unit[par] = claim_next(a.sched);  // next, in flight
       int64_t o;
       Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
       v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
@@ -275,7 +349,10 @@ __global__ void __launch_bounds__(BLOCK) seg_kernel(SegArgs a) {
 }
 
 // ------------------------------------------------------------- stream kernel
-// R and long-row KR shapes (C == 1): each unit is one contiguous range.  Its
+// R and long-row KR shapes (C == 1): each unit is one contiguous range; RKR
+// with 16-B aligned rows (C > 1): each unit is a run of whole rows of one
+// output at the row stride, and the stages are filled from the rows'
+// concatenation (a fold does not care where a row ends).  The unit's
 // 16-B-aligned body is streamed into a ring of NS shared-memory stages by the
 // TMA bulk-copy engine (cp.async.bulk, completion on an mbarrier with a byte
 // count); thread 0 is the producer and keeps NS stages (NS*STAGE bytes) in
@@ -292,6 +369,17 @@ template <typename T>
 __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u) {
   constexpr int VEC = 16 / sizeof(T);
   StreamGeom g;
+  if (a.C > 1) {  // RKR: whole 16-B aligned rows r0..r1-1 of output o (plan), no head / tail
+    const int64_t S = a.Sr;
+    g.o = u / S;
+    const int64_t s = u - g.o * S;
+    const int64_t r0 = split_lo(a.C, S, s), r1 = split_lo(a.C, S, s + 1);
+    g.row = static_cast<const T*>(a.in) + g.o * a.oStride + r0 * a.rowStride;
+    g.head = 0;
+    g.tail = 0;
+    g.nbody = (r1 - r0) * a.L;
+    return g;
+  }
   const int64_t S = a.Sc;
   g.o = u / S;
   const int64_t s = u - g.o * S;
@@ -308,7 +396,7 @@ __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u)
 }
 
 template <int OP, typename T, int NS, int STAGE>
-__global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
+__global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant__ SegArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -324,7 +412,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
-  const int64_t S = a.Sc;
+  const int64_t S = a.Sr * a.Sc;
   const bool whole = (a.O == 1);
 
   if (tid == 0) {
@@ -344,9 +432,9 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = (long long)atomicAdd(a.sched, 1ull);
+      long long u = claim_first();
       while (true) {
-        const long long nu = (long long)atomicAdd(a.sched, 1ull);  // next claim, in flight
+        const long long nu = claim_next(a.sched);  // next claim, in flight
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < a.units ? u : -1;
         ++seq;
@@ -359,12 +447,23 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
         const char* src = static_cast<const char*>(geo.row) + geo.head * (int64_t)sizeof(T);
         const int64_t bytes = geo.nbody * (int64_t)sizeof(T);
         const int64_t nk = (bytes + STAGE - 1) / STAGE;
+        // RKR units are several rows at a stride: each stage is filled from
+        // the concatenation of the unit's rows (one bulk copy per row piece)
+        const int64_t rb = a.C > 1 ? a.L * (int64_t)sizeof(T) : bytes;
+        const int64_t rs = a.rowStride * (int64_t)sizeof(T);
+        int64_t r = 0, inrow = 0;
         for (int64_t k = 0; k < nk; ++k, ++g) {
           const int slot = (int)(g % NS);
           if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
           const unsigned nb = (unsigned)min((int64_t)STAGE, bytes - k * STAGE);
           mbar_expect_tx(&full[slot], nb);
-          bulk_g2s(stage_mem + slot * STAGE, src + k * STAGE, nb, &full[slot]);
+          for (unsigned done = 0; done < nb;) {
+            const unsigned len = (unsigned)min((int64_t)(nb - done), rb - inrow);
+            bulk_g2s(stage_mem + slot * STAGE + done, src + r * rs + inrow, len, &full[slot]);
+            done += len;
+            inrow += len;
+            if (inrow == rb) { inrow = 0; ++r; }
+          }
         }
         u = nu;
       }
@@ -453,7 +552,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(SegArgs a) {
     cons_sync();
     if (s_last) {
       __threadfence();
-      Acc w = fold_partials<OP, T>(partials, S, ct, kConsThreads);
+      Acc w = fold_partials_vec<OP, T>(partials, S, ct, kConsThreads);
       w = cons_reduce<OP, T>(w, smem, cw, lane);
       if (ct == 0) {
         const T r = merge_init<OP, T>(w, out, 0, a.init_from_out);
@@ -508,9 +607,9 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = (long long)atomicAdd(a.sched, 1ull);
+      long long u = claim_first();
       while (true) {
-        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < S ? u : -1;
         ++seq;
@@ -599,7 +698,7 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
 // left 1/2 to 31/32 of its lanes idle on such rows (r01: 1 TB/s on the
 // paper's 2^20 x 2 x 32 gang case).
 template <int OP, typename T>
-__global__ void __launch_bounds__(kBlock) colflat_kernel(ColArgs a) {
+__global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __grid_constant__ ColArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -747,34 +846,36 @@ __global__ void __launch_bounds__(kBlock) colflat_kernel(ColArgs a) {
 
 // ------------------------------------------------------------- RKR rows kernel
 // RKR (reduce outer k and inner i, keep the middle j) with short rows
-// (row_bytes = L*size a power of two in [512 B, 2 KiB], 16-B aligned): the
-// rows (k, j) are contiguous in memory and row r feeds output j = r mod K, so
-// the whole nest is streamed like the rows kernel (producer warp, bulk copies
-// of 16 KiB stages); each consumer warp reduces its rows (a2) and lane 0
-// folds the result into a shared per-output array acc[K] (a3) -- rows in
-// flight never share an output because K >= 32 >= rows per stage x stages.
-// A unit (a block of whole stages) leaves a K-wide partial row; the gang tier
-// is two-level (unit partials -> groups of kGroupFold -> outputs).
-
+// (row_bytes = L*size a power of two in [512 B, 2 KiB], 16-B aligned).  For a
+// fixed k the rows (k, j) are contiguous, so J = 16 KiB / row_bytes
+// consecutive outputs j form one 16 KiB stage.  A unit is (j-block jb, range
+// of k): the producer warp streams the unit's stages (one cp.async.bulk per
+// k, K*row_bytes apart in memory), and consumer warp w always
+// meets the same rows -- outputs jb*J + w*rpw .. + rpw-1 -- in every stage,
+// so its lanes accumulate them in registers across the whole k range with no
+// shared-memory combine and no barrier per stage (the rows kernel's layout
+// with a k loop).  At the end of a unit each warp reduces its rows (a2) and
+// runs the per-output gang tier (a4): partials[j][s], a ticket per output,
+// the last unit of output j folds its S partials.  (A first version streamed
+// all rows and folded them by j into K-wide shared-memory partial rows: 0.60
+// of peak, latency bound on the partial-row folds, r01.)
 template <int OP, typename T, int NS>
-__global__ void __launch_bounds__(kWsBlock) rkr_kernel(RkrArgs a) {
+__global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ RkrArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
   constexpr int STAGE = kStageBytes;
   constexpr int RING = 8;
-  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE, then acc[K]
+  extern __shared__ __align__(1024) unsigned char stage_mem[];  // NS * STAGE
   __shared__ __align__(8) uint64_t full[NS];
   __shared__ __align__(8) uint64_t empty[NS];
   __shared__ long long s_units[RING];
-  __shared__ int s_last;
-  Acc* acc = reinterpret_cast<Acc*>(stage_mem + NS * STAGE);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   const int64_t row_bytes = a.L * (int64_t)sizeof(T);
-  const int rshift = __ffsll(row_bytes) - 1;
-  const int rps = (int)(STAGE >> rshift);
-  const int64_t nst = (a.NR + rps - 1) / rps;
+  const int rshift = __ffsll(row_bytes) - 1;  // row_bytes is a power of two
+  const int J = (int)(STAGE >> rshift);        // rows (outputs) per stage: 8, 16 or 32
+  const int64_t S = a.S;                       // k splits per j-block
 
   if (tid == 0) {
 #pragma unroll
@@ -790,25 +891,27 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(RkrArgs a) {
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = (long long)atomicAdd(a.sched, 1ull);
+      long long u = claim_first();
       while (true) {
-        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
-        s_units[seq & (RING - 1)] = u < a.S ? u : -1;
+        s_units[seq & (RING - 1)] = u < a.units ? u : -1;
         ++seq;
-        if (u >= a.S) {
+        if (u >= a.units) {
           if (g >= NS) mbar_wait(&empty[slot0], (unsigned)(((g / NS) - 1) & 1));
           mbar_arrive(&full[slot0]);
           break;
         }
-        const int64_t st0 = split_lo(nst, a.S, u), st1 = split_lo(nst, a.S, u + 1);
-        for (int64_t st = st0; st < st1; ++st, ++g) {
+        const int64_t jb = u / S, s = u - jb * S;
+        const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
+        const unsigned nb = (unsigned)(min((int64_t)J, a.K - jb * J) << rshift);
+        const char* src = static_cast<const char*>(a.in) + ((k0 * a.K + jb * J) << rshift);
+        const int64_t kstride = a.K << rshift;  // bytes between consecutive k
+        for (int64_t k = k0; k < k1; ++k, ++g, src += kstride) {
           const int slot = (int)(g % NS);
           if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
-          const int64_t row0 = st * rps;
-          const unsigned nb = (unsigned)(min((int64_t)rps, a.NR - row0) << rshift);
           mbar_expect_tx(&full[slot], nb);
-          bulk_g2s(stage_mem + slot * STAGE, static_cast<const char*>(a.in) + (row0 << rshift), nb, &full[slot]);
+          bulk_g2s(stage_mem + slot * STAGE, src, nb, &full[slot]);
         }
         u = nu;
       }
@@ -818,105 +921,77 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(RkrArgs a) {
   }
 
   // ---------------- consumer warps
-  const int ct = tid - 32, cw = warp - 1;
+  const int cw = warp - 1;
+  const int rpw = J / kConsWarps;          // rows per warp per stage (1, 2 or 4)
+  const int vpl = (int)(row_bytes >> 9);   // 16-B vectors per lane per row (1, 2 or 4)
   Acc* partials = static_cast<Acc*>(a.partials);
-  Acc* P2 = partials + a.S * a.K;
   int seq = 0;
   int64_t g = 0;
-  // fold rows [0, n) of a [n][K] partial block into column c (all consumers)
-  auto fold_col = [&](const Acc* src, int64_t n, int64_t c) {
-    Acc z = O::identity();
-    int64_t r = 0;
-    for (; r + 3 < n; r += 4) {
-      Acc y[4];
-#pragma unroll
-      for (int k = 0; k < 4; ++k) y[k] = ld_partial(src + (r + k) * a.K + c);
-#pragma unroll
-      for (int k = 0; k < 4; ++k) z = O::combine(z, y[k]);
-    }
-    for (; r < n; ++r) z = O::combine(z, ld_partial(src + r * a.K + c));
-    return z;
-  };
   while (true) {
     mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
-    for (int64_t c = ct; c < a.K; c += kConsThreads) acc[c] = O::identity();
-    cons_sync();
-    const int64_t st0 = split_lo(nst, a.S, u), st1 = split_lo(nst, a.S, u + 1);
-    for (int64_t st = st0; st < st1; ++st, ++g) {
+    const int64_t jb = u / S, s = u - jb * S;
+    const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
+    const int nrows = (int)min((int64_t)J, a.K - jb * J);
+    Acc acc[4][VEC];
+#pragma unroll
+    for (int rr = 0; rr < 4; ++rr)
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[rr][q] = O::identity();
+    for (int64_t k = k0; k < k1; ++k, ++g) {
       const int slot = (int)(g % NS);
-      if (st > st0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
-      const int64_t row0 = st * rps;
-      const int nrows = (int)min((int64_t)rps, a.NR - row0);
+      if (k > k0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const unsigned char* sm = stage_mem + slot * STAGE;
-      const int rpw = rps / kConsWarps;
-      const int vpl = (int)(row_bytes >> 9);
-      Acc v[4];
 #pragma unroll
       for (int rr = 0; rr < 4; ++rr) {
-        v[rr] = O::identity();
         const int r = cw * rpw + rr;
         if (rr < rpw && r < nrows) {
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            if (k < vpl) {
-              const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + (k * 32 + lane) * 16);
+          for (int kk = 0; kk < 4; ++kk) {
+            if (kk < vpl) {
+              const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + (kk * 32 + lane) * 16);
 #pragma unroll
-              for (int q = 0; q < VEC; ++q) v[rr] = O::combine(v[rr], O::lift(unpack<T>(x, q)));
+              for (int q = 0; q < VEC; ++q) acc[rr][q] = O::combine(acc[rr][q], O::lift(unpack<T>(x, q)));
             }
           }
         }
       }
-      fence_proxy_async_smem();
+      fence_proxy_async_smem();  // generic reads before the async refill
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[slot]);
+      if (lane == 0) mbar_arrive(&empty[slot]);  // the stage is consumed into registers
+    }
 #pragma unroll
-      for (int rr = 0; rr < 4; ++rr) {
-        if (rr < rpw) {
-          const Acc w = group_reduce<OP, T, 32>(v[rr]);
-          const int r = cw * rpw + rr;
-          if (lane == 0 && r < nrows) {
-            const int64_t j = (row0 + r) % a.K;
-            acc[j] = O::combine(acc[j], w);
+    for (int rr = 0; rr < 4; ++rr) {
+      const int r = cw * rpw + rr;
+      if (rr < rpw && r < nrows) {  // warp-uniform
+        Acc v = acc[rr][0];
+#pragma unroll
+        for (int q = 1; q < VEC; ++q) v = O::combine(v, acc[rr][q]);
+        v = group_reduce<OP, T, 32>(v);
+        const int64_t o = jb * J + r;
+        if (S == 1) {
+          if (lane == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+        } else {  // a4: the last unit of output o folds its S partials in split order
+          int last = 0;
+          if (lane == 0) {
+            partials[o * S + s] = v;
+            __threadfence();
+            last = (atomicAdd(&a.tickets[o], 1u) == (unsigned)(S - 1));
+          }
+          last = __shfl_sync(0xffffffffu, last, 0);
+          if (last) {
+            __threadfence();
+            Acc w = fold_partials<OP, T>(partials + o * S, S, lane, 32);
+            w = group_reduce<OP, T, 32>(w);
+            if (lane == 0) {
+              out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+              a.tickets[o] = 0u;
+            }
           }
         }
       }
     }
-    cons_sync();  // acc[] complete for this unit
-    // a4, two levels: unit partial row -> group -> outputs
-    for (int64_t c = ct; c < a.K; c += kConsThreads) partials[u * a.K + c] = acc[c];
-    const int64_t gi = u / kGroupFold, g0 = gi * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
-    cons_sync();
-    if (ct == 0) {
-      __threadfence();
-      s_last = (atomicAdd(&a.tickets[gi], 1u) == (unsigned)(gsz - 1));
-    }
-    cons_sync();
-    if (s_last) {
-      __threadfence();
-      if (a.G2 == 1) {
-        for (int64_t c = ct; c < a.K; c += kConsThreads)
-          out[c] = merge_init<OP, T>(fold_col(partials + g0 * a.K, gsz, c), out, c, a.init_from_out);
-        if (ct == 0) a.tickets[gi] = 0u;
-      } else {
-        for (int64_t c = ct; c < a.K; c += kConsThreads) P2[gi * a.K + c] = fold_col(partials + g0 * a.K, gsz, c);
-        cons_sync();
-        if (ct == 0) {
-          a.tickets[gi] = 0u;
-          __threadfence();
-          s_last = (atomicAdd(&a.tickets[a.G2], 1u) == (unsigned)(a.G2 - 1));
-        }
-        cons_sync();
-        if (s_last) {
-          __threadfence();
-          for (int64_t c = ct; c < a.K; c += kConsThreads)
-            out[c] = merge_init<OP, T>(fold_col(P2, a.G2, c), out, c, a.init_from_out);
-          if (ct == 0) a.tickets[a.G2] = 0u;
-        }
-      }
-    }
-    cons_sync();
     ++seq;
   }
 }
@@ -926,7 +1001,11 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(RkrArgs a) {
 // the CTA's warps stride over the reduced rows of a row chunk; the worker tier
 // is a cross-warp combine of per-column partials in shared memory.
 template <int OP, typename T, int VEC, int BLOCK, int U>
-__global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
+// (the column kernel keeps its 16-B loads batched with min 1, not 4 -- SASS guard)
+#ifndef XR_COL_MINB
+#define XR_COL_MINB 1
+#endif
+__global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_constant__ ColArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int NW = BLOCK / 32;
@@ -941,12 +1020,12 @@ __global__ void __launch_bounds__(BLOCK) col_kernel(ColArgs a) {
   const int64_t per_b = a.tiles * a.S;
 
   __shared__ long long s_unit[2];
-  if (t == 0) s_unit[0] = (long long)atomicAdd(a.sched, 1ull);
+  if (t == 0) s_unit[0] = claim_first();
   __syncthreads();
   long long u = s_unit[0];
   int par = 1;
   while (u < a.units) {
-    if (t == 0) s_unit[par] = (long long)atomicAdd(a.sched, 1ull);  // next unit, in flight
+    if (t == 0) s_unit[par] = claim_next(a.sched);  // next unit, in flight
     const int64_t b = u / per_b, rem = u - b * per_b;
     const int64_t tile = rem / a.S, s = rem - tile * a.S;
     const int64_t col = tile * TW + (int64_t)lane * VEC;
@@ -1100,9 +1179,9 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = (long long)atomicAdd(a.sched, 1ull);
+      long long u = claim_first();
       while (true) {
-        const long long nu = (long long)atomicAdd(a.sched, 1ull);
+        const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < a.units ? u : -1;
         ++seq;
@@ -1340,13 +1419,11 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
     }
     case K_RKR: {
       auto kern = rkr_kernel<OP, T, kStages>;
-      const int dyn = kStages * kStageBytes + (int)(p.rkr.K * sizeof(typename Op<OP, T>::Acc));
+      constexpr int dyn = kStages * kStageBytes;
       static int occ = [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kStages * kStageBytes + 16384);
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, kStages * kStageBytes + 16384) !=
-                cudaSuccess || n < 1)
-          n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
         return n;
       }();
       int64_t grid = grid_for(p.units, num_sms, occ);

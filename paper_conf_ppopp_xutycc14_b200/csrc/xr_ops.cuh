@@ -23,6 +23,21 @@ template <typename T> __device__ __forceinline__ T ld_scalar(const T* p) { retur
 
 // L2-coherent load of a partial written by another CTA of the same grid.
 template <typename A> __device__ __forceinline__ A ld_partial(const A* p) { return __ldcg(p); }
+// 16 B of partials, L2-coherent (ld.global.cg)
+__device__ __forceinline__ U128 ld_partial16(const void* p) {
+  U128 r;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.w[0]), "=r"(r.w[1]), "=r"(r.w[2]), "=r"(r.w[3])
+               : "l"(p));
+  return r;
+}
+// q-th accumulator packed in a 16-B vector (4-B or 8-B accumulators)
+template <typename A> __device__ __forceinline__ A acc_at(const U128& u, int q) {
+  A a;
+  if constexpr (sizeof(A) == 4) memcpy(&a, &u.w[q], 4);
+  else { const uint32_t lohi[2] = {u.w[2 * q], u.w[2 * q + 1]}; memcpy(&a, lohi, 8); }
+  return a;
+}
 
 template <typename T> __device__ __forceinline__ T unpack(const U128& u, int q) {
   static_assert(sizeof(T) == 4 || sizeof(T) == 8, "dtype");
@@ -124,6 +139,12 @@ namespace xr {
 // Dynamic unit claiming for CTA-wide work: thread 0 fetches the next unit
 // index (prefetched one unit ahead into a parity slot) from a device counter;
 // the last CTA to exit resets the counters for the next launch.
+// The first unit of every CTA is static (blockIdx.x): the first dynamic claim
+// would put an L2 atomic round trip before the first load of every CTA.
+__device__ __forceinline__ long long claim_first() { return (long long)blockIdx.x; }
+__device__ __forceinline__ long long claim_next(unsigned long long* c) {
+  return (long long)gridDim.x + (long long)atomicAdd(c, 1ull);
+}
 __device__ __forceinline__ void sched_exit(unsigned long long* c) {
   if (threadIdx.x == 0) {
     __threadfence();

@@ -228,32 +228,37 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   else { O = run_n[1]; C = run_n[0]; L = run_n[2]; rowStride = O * L; oStride = L; p->shape = XR_SHAPE_RKR; }
 
   const int64_t row_bytes = L * size;
-  // RKR with short rows: stream all rows, fold by output in shared memory.
-  // OPT-IN (XR_RKR=1): measured r01 on 512^3 int32/fp32 GV at 0.60 of peak vs
-  // 0.82 for the seg path -- its K-wide partial-row folds are latency bound.
-  if (!seg_only && !seg_only_small && nr == 3 && std::getenv("XR_RKR") != nullptr &&
-      row_bytes >= 512 && row_bytes <= 2048 &&
-      (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= 32 && O * asz <= 16384 &&
-      std::getenv("XR_NO_BULK") == nullptr) {
-    const int64_t rps = kStageBytes / row_bytes;
-    const int64_t NR = C * O;
-    const int64_t nst = cdiv(NR, rps);
-    const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;
-    const int64_t k = 2;  // equal units per CTA
-    int64_t S = std::max<int64_t>(1, std::min<int64_t>(nst / kStages, k * cap));
-    if (chain_capped) S = std::max<int64_t>(S, cdiv(NR, (int64_t)kChainCap * 8));
-    const int64_t G2 = cdiv(S, kGroupFold);
+  // RKR with short rows (power-of-two row_bytes in [512 B, 2 KiB], 16-B
+  // aligned, at least one full 16 KiB j-block): the rkr rows kernel -- units
+  // are (block of J = 16 KiB / row_bytes outputs, range of k), each stage one
+  // bulk copy of J contiguous rows, accumulated per warp in registers.
+  if (!seg_only && !seg_only_small && nr == 3 && row_bytes >= 512 && row_bytes <= 2048 &&
+      (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= kStageBytes / row_bytes &&
+      std::getenv("XR_NO_RKR") == nullptr && std::getenv("XR_NO_BULK") == nullptr) {
+    const int64_t J = kStageBytes / row_bytes;
+    const int64_t njb = cdiv(O, J);
+    const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;  // resident CTAs (64 KiB ring each)
+    const char* eu = std::getenv("XR_RKR_UNITS_PER_CTA");   // tuning override
+    // r01 sweep (512^3 32-bit GV): 4 units per CTA 0.89, 8 0.91, 16 0.81, 32 0.82
+    const int64_t k = eu ? std::max(1, std::atoi(eu)) : 8;
+    // k units per resident CTA, each >= kStages stages (k values)
+    int64_t S = std::max<int64_t>(1, std::min<int64_t>(cdiv(k * cap, njb), C / kStages));
+    // fp32 '+': each lane accumulator folds vpl elements per k (chains <= kChainCap)
+    if (chain_capped) S = std::max<int64_t>(S, cdiv(C * (row_bytes >> 9), (int64_t)kChainCap));
+    S = std::max<int64_t>(1, std::min<int64_t>(S, C));
     p->kernel = K_RKR;
     p->group = 32;
     p->vec = vec;
     p->splits = S;
-    p->units = S;
+    p->units = njb * S;
     p->sched = true;
-    p->grid_hint = std::min<int64_t>(cap, cdiv(S, k));
-    p->ws_bytes = (S + G2) * O * asz;
-    p->tickets = G2 + 1;
+    p->grid_hint = std::min<int64_t>(cap, p->units);
+    if (S > 1) {
+      p->ws_bytes = O * S * asz;
+      p->tickets = O;
+    }
     RkrArgs& r = p->rkr;
-    r.K = O; r.L = L; r.NR = NR; r.S = S; r.G2 = G2;
+    r.K = O; r.L = L; r.C = C; r.S = S; r.units = p->units;
     return;
   }
   // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
@@ -264,8 +269,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int64_t rps = kStageBytes / row_bytes;
     const int64_t nst = cdiv(O, rps);
     const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;
-    const int64_t k = 2;  // equal units per CTA (see the column kernel)
-    const int64_t units = std::max<int64_t>(1, std::min<int64_t>(nst / kStages, k * cap));
+    // many short units: a unit boundary costs the rows kernel nothing (no
+    // epilogue, the producer streams across it), and short units balance the
+    // tail (r01 sweep, 512^3 32-bit V: 2 units per CTA 0.91 of peak, 8 0.95,
+    // 32 1.00)
+    const char* eu = std::getenv("XR_ROWS_UNITS_PER_CTA");  // tuning override
+    const int64_t k = eu ? std::max(1, std::atoi(eu)) : 32;
+    const int64_t units = std::max<int64_t>(1, std::min<int64_t>(nst, k * cap));
     p->kernel = K_ROWS;
     p->group = 32;
     p->vec = vec;
@@ -294,17 +304,28 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // long contiguous rows (R, KR): the bulk-copy stream kernel; every unit must
   // cover at least kStages stages so the producer stays <= 3 units ahead
   const int64_t stage_elems = kStageBytes / size;
-  const bool stream = !seg_only && !seg_only_small && C == 1 && row_bytes >= (int64_t)kStages * kStageBytes &&
-                      std::getenv("XR_NO_BULK") == nullptr;
+  // RKR with 16-B aligned rows of >= 4 KiB: the same kernel streams each
+  // unit's rows (one bulk copy per row piece).  r01 sweep on 512^3 GV: 64-bit
+  // (4 KiB rows) 0.95-1.01 of peak vs 0.66-0.95 for the seg kernel; 32-bit
+  // (2 KiB rows) no better than seg (0.83-0.87 both), so those stay on seg.
+  const char* rkr_min = std::getenv("XR_RKR_STREAM_MIN_ROW");  // tuning override (bytes)
+  const bool rkr_stream = nr == 3 && row_bytes >= (rkr_min ? std::atoll(rkr_min) : 4096) &&
+                          row_bytes % 16 == 0 && in_addr % 16 == 0 && std::getenv("XR_NO_RKR_STREAM") == nullptr;
+  const bool stream = !seg_only && !seg_only_small && std::getenv("XR_NO_BULK") == nullptr &&
+                      ((C == 1 && row_bytes >= (int64_t)kStages * kStageBytes) || rkr_stream);
   if (stream) {
-    const int64_t min_stages = O == 1 ? kStages : 4 * kStages;  // several outputs: amortise the epilogue
+    // several outputs: amortise the epilogue (RKR: 512 KiB units, r01 sweep)
+    const int64_t min_stages = O == 1 ? kStages : C > 1 ? 8 * kStages : 4 * kStages;
     S = std::min<int64_t>(S, std::max<int64_t>(1, work / (min_stages * stage_elems)));
   }
   // fp32 '+': per-thread chains <= kChainCap (stream: 16 accumulators per thread)
   if (chain_capped) S = std::max<int64_t>(S, cdiv(work, (int64_t)kChainCap * W * vec * kUnroll));
+  if (stream && std::getenv("XR_STREAM_SPLITS") != nullptr)  // tuning override
+    S = std::max<int64_t>(1, std::atoll(std::getenv("XR_STREAM_SPLITS")));
+  if (stream) W = kBlock;  // CTA-wide units, claimed dynamically
   if (S > 1 && W < 32) W = 32;  // the gang-tier ticket runs per warp or per CTA
   int64_t Sr, Sc;
-  if (C >= S) { Sr = S; Sc = 1; }
+  if (C >= S || (stream && C > 1)) { Sr = std::min(S, C); Sc = 1; }  // stream RKR units are whole rows
   else { Sr = C; Sc = std::min<int64_t>(cdiv(S, C), std::max<int64_t>(1, L / vec)); }
   S = Sr * Sc;
 

@@ -148,7 +148,7 @@ def test_plan_fp32_chain_cap(xr, case):
     _, dims, lv = case
     p = xr.xr_plan_describe("+", "fp32", dims, lv, 256)
     if p["kernel"] == "rkr":
-        per_acc = p["cdims"][0] * p["cdims"][2] / p["splits"] / 32  # per lane: rows x VEC per unit
+        per_acc = p["cdims"][0] * p["cdims"][2] / p["splits"] / (32 * p["vec"])  # per lane accumulator: k range x vectors per row
     elif p["kernel"] == "rows":
         per_acc = p["cdims"][1] / (32 * p["vec"])  # one row per warp-wide fold, VEC chains per lane
     elif p["kernel"] in ("seg", "stream"):

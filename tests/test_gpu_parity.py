@@ -365,17 +365,52 @@ def test_colflat_narrow_rows(dtype, row_bytes, staging):
 
 @pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
 @pytest.mark.parametrize("row_bytes", [512, 1024, 2048])
-def test_rkr_kernel_short_rows(dtype, row_bytes, monkeypatch):
-    """RKR (gang + vector reduced, worker kept) with short rows: the bulk-
-    streamed rows folded by their middle index (forced with XR_SMALL_BYTES=0)."""
+@pytest.mark.parametrize("units", ["auto", "1", "64"])
+def test_rkr_kernel_short_rows(dtype, row_bytes, units, monkeypatch):
+    """RKR (gang + vector reduced, worker kept) with short rows: the rkr rows
+    kernel (j-blocks of 16 KiB / row_bytes outputs streamed per k, per-warp
+    register accumulation, per-output gang tier), forced with XR_SMALL_BYTES=0;
+    ragged j-blocks (K not a multiple of the block), k split from 1 unit per
+    CTA (few long units) to 64, with init."""
     import paper_conf_ppopp_xutycc14_b200 as xr
     monkeypatch.setenv("XR_SMALL_BYTES", "0")
-    monkeypatch.setenv("XR_RKR", "1")  # opt-in kernel (DESIGN.md: slower than seg on 512^3)
+    if units != "auto":
+        monkeypatch.setenv("XR_RKR_UNITS_PER_CTA", units)
     L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
-    for R1, K, op in [(7, 32, "+"), (33, 100, "max"), (5, 999, "&&"), (300, 40, "*")]:
+    for R1, K, op in [(7, 32, "+"), (33, 100, "max"), (5, 999, "&&"), (300, 40, "*"), (64, 37, "||"),
+                      (1, 64, "min")]:
         dims = (R1, K, L)
         x = recipes.make(KIND[op], dims, oracle.mask_of("gv"), dtype, R1 * K)
         init = recipes.make("ints", (K, 1, 1), 1, dtype, 4)
         check(op, dtype, dims, "gv", gpu_reduce(op, dtype, dims, "gv", x, init=init), x, init=init)
-        if K * (8 if dtype == "int64" or dtype == "fp64" else 4) <= 16384:
+        if R1 > 1:
             assert xr.xr_plan_describe(op, dtype, dims, "gv", 256)["kernel"] == "rkr"
+        if dtype.startswith("int"):
+            xb = recipes.make("bxor", dims, oracle.mask_of("gv"), dtype, R1 + K)
+            check("^", dtype, dims, "gv", gpu_reduce("^", dtype, dims, "gv", xb), xb)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [1024, 1536, 2048, 4096, 20480])
+@pytest.mark.parametrize("splits", ["auto", "1", "3", "7"])
+def test_stream_rkr_rows(dtype, row_bytes, splits, monkeypatch):
+    """RKR (gang + vector reduced, worker kept) with 16-B aligned rows of >= 1 KiB:
+    the stream kernel fills its stages from each unit's rows at the row stride
+    (rows straddling stages when row_bytes does not divide 16 KiB, rows longer
+    than a stage); ragged row splits (XR_STREAM_SPLITS), with init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    monkeypatch.setenv("XR_RKR_STREAM_MIN_ROW", "1024")  # the planner's default is 4 KiB rows
+    monkeypatch.setenv("XR_NO_RKR", "1")  # 1-2 KiB rows would take the rkr rows kernel
+    if splits != "auto":
+        monkeypatch.setenv("XR_STREAM_SPLITS", splits)
+    L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for R1, K, op in [(7, 3, "+"), (33, 100, "max"), (5, 129, "&&"), (61, 8, "*"), (19, 17, "||")]:
+        dims = (R1, K, L)
+        x = recipes.make(KIND[op], dims, oracle.mask_of("gv"), dtype, R1 * K + row_bytes)
+        init = recipes.make("ints", (K, 1, 1), 1, dtype, 4)
+        check(op, dtype, dims, "gv", gpu_reduce(op, dtype, dims, "gv", x, init=init), x, init=init)
+        assert xr.xr_plan_describe(op, dtype, dims, "gv", 256)["kernel"] == "stream"
+        if dtype.startswith("int"):  # & | ^ on the same path
+            xb = recipes.make("bxor", dims, oracle.mask_of("gv"), dtype, R1 + K)
+            check("^", dtype, dims, "gv", gpu_reduce("^", dtype, dims, "gv", xb), xb)

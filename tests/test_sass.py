@@ -1,0 +1,29 @@
+"""SASS guard (CPU only): the register kernels' fold loops keep >= 4 16-B
+loads in flight per thread.  ptxas once sank the unrolled loads of fold_row
+next to their uses in some instantiations (2 loads in flight; fp64 && || rows
+fell to 0.63 of peak), which no parity test can see -- DESIGN.md section 6."""
+import importlib.util
+import os
+import shutil
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+SO = os.path.join(ROOT, "paper_conf_ppopp_xutycc14_b200", "libxreduce.so")
+
+
+def _checker():
+    spec = importlib.util.spec_from_file_location("sass_ldg_check", os.path.join(ROOT, "tools", "sass_ldg_check.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    return mod
+
+
+@pytest.mark.skipif(shutil.which("cuobjdump") is None, reason="cuobjdump not on PATH")
+def test_fold_loops_keep_four_loads_in_flight():
+    got = _checker().batches(SO)
+    fams = ("xr::seg_kernel<", "xr::col_kernel<", "xr::colflat_kernel<")
+    checked = {n: b for n, (b, cnt) in got.items() if n.startswith(tuple("void " + f for f in fams)) and cnt >= 4}
+    assert len(checked) >= 150, len(checked)  # every (op, dtype, group) instantiation
+    bad = {n: b for n, b in checked.items() if b < 4}
+    assert not bad, bad

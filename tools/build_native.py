@@ -50,7 +50,11 @@ def _stale(obj: str, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, ptxas_verbose: bool = False, quiet: bool = True) -> str:
+def build(force: bool = False, ptxas_verbose: bool = False, quiet: bool = True,
+          defines=(), so_path: str | None = None, obj_dir: str | None = None) -> str:
+    """defines / so_path / obj_dir: A/B variants (tools/build_native.py --variant)."""
+    OBJ = obj_dir or globals()["OBJ"]
+    SO = so_path or globals()["SO"]
     os.makedirs(OBJ, exist_ok=True)
     nccl = _nccl_dir()
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", os.path.join(nccl, "include")]
@@ -63,7 +67,7 @@ def build(force: bool = False, ptxas_verbose: bool = False, quiet: bool = True) 
         objs.append(obj)
         if force or _stale(obj, [src] + hdr):
             cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
-                   "--expt-relaxed-constexpr", "-c", src, "-o", obj, *inc]
+                   "--expt-relaxed-constexpr", *["-D" + d for d in defines], "-c", src, "-o", obj, *inc]
             if ptxas_verbose:
                 cmd += ["-Xptxas", "-v"]
             jobs.append(cmd)
@@ -111,5 +115,12 @@ def build_devapi_test(force: bool = False) -> str:
 
 
 if __name__ == "__main__":
+    if "--variant" in sys.argv:  # A/B build: variants/libxreduce_<name>.so with -D defines
+        i = sys.argv.index("--variant")
+        name, defs = sys.argv[i + 1], [a[2:] for a in sys.argv[i + 2:] if a.startswith("-D")]
+        vdir = os.path.join(ROOT, "variants")
+        print(build(force=True, defines=defs, so_path=os.path.join(vdir, f"libxreduce_{name}.so"),
+                    obj_dir=os.path.join(vdir, "obj_" + name)))
+        sys.exit(0)
     print(build(force="--force" in sys.argv, ptxas_verbose="--ptxas-v" in sys.argv, quiet=False))
     print(build_devapi_test(force="--force" in sys.argv))

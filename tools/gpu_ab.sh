@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 OUT=gpurun_out/ab_${TAG:-x}.jsonl
 : > $OUT
-CELLS=${CELLS:-"cfg5-+-int32-gwv cfg5-||-fp64-v cfg5-&&-fp64-gv cfg5-|-int32-wv cfg5-+-int32-v cfg2-f32-sum"}
+CELLS=${CELLS:-"cfg5-add-int32-gwv cfg5-lor-fp64-v cfg5-land-fp64-gv cfg5-or-int32-wv cfg5-add-int32-v cfg2-f32-sum"}
 for rep in 1 2; do
   for t in new old; do
     if [ $t = new ]; then D=.; else D=$AB_DIR; fi

@@ -4,7 +4,9 @@
   python tools/kdriver.py CASE [--reps R] [--time]
 
 CASE names a BASELINE config shape, e.g. cfg2-f32-sum, cfg2-i64-sum, cfg3-row,
-cfg3-col, cfg4-heat, cfg5-<op>-<dtype>-<mask>, cfg1-<mask>.  Inputs are random
+cfg3-col, cfg4-heat, cfg5-<op>-<dtype>-<mask>, cfg1-<mask>, or any nest
+nest-<op>-<dtype>-<n0>x<n1>x<n2>-<mask>.  --cold flushes L2 (a 256 MiB write)
+before every timed call (cfg1 "cold" latency).  Inputs are random
 device tensors (values do not change the memory traffic).  With --time, prints
 a JSON line per case with the CUDA-event kernel time, algorithmic bytes and
 GB/s vs the measured HBM peak.
@@ -57,6 +59,11 @@ def cases(name):
         op = {"mul": "*", "and": "&", "or": "|", "xor": "^", "land": "&&", "lor": "||", "add": "+",
               "max": "max", "min": "min"}[op]
         return [(name, op, dtype, (512, 512, 512), lv)]
+    if name.startswith("nest-"):  # nest-<op>-<dtype>-<n0>x<n1>x<n2>-<mask>, op as in cfg5
+        _, op, dtype, dims, lv = name.split("-")
+        op = {"mul": "*", "and": "&", "or": "|", "xor": "^", "land": "&&", "lor": "||", "add": "+",
+              "max": "max", "min": "min"}[op]
+        return [(name, op, dtype, tuple(int(d) for d in dims.split("x")), lv)]
     raise SystemExit(f"unknown case {name}")
 
 
@@ -67,7 +74,17 @@ def peak():
         return 6650.0
 
 
-def run_reduce(label, op, dtype, dims, lv, reps, timed, cache):
+_FLUSH = None
+
+
+def flush_l2():
+    global _FLUSH
+    if _FLUSH is None:
+        _FLUSH = torch.empty(64 << 20, dtype=torch.float32, device="cuda")  # 256 MiB > 126 MB L2
+    _FLUSH.fill_(1.0)
+
+
+def run_reduce(label, op, dtype, dims, lv, reps, timed, cache, cold=False):
     n = dims[0] * dims[1] * dims[2]
     key = (dtype, n)
     if key not in cache:
@@ -83,6 +100,8 @@ def run_reduce(label, op, dtype, dims, lv, reps, timed, cache):
     torch.cuda.synchronize()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     for a, b in evs:
+        if cold:
+            flush_l2()
         a.record(s)
         xr.xr_reduce(op, dtype, dims, lv, x.data_ptr(), out.data_ptr(), s.cuda_stream)
         b.record(s)
@@ -92,7 +111,7 @@ def run_reduce(label, op, dtype, dims, lv, reps, timed, cache):
         med = ms[len(ms) // 2]
         byts = (n + cnt) * SIZE[dtype]
         plan = xr.xr_plan_describe(op, dtype, dims, lv, x.data_ptr())
-        print(json.dumps({"case": label, "op": op, "dtype": dtype, "dims": dims, "levels": lv,
+        print(json.dumps({"case": label + ("-cold" if cold else ""), "op": op, "dtype": dtype, "dims": dims, "levels": lv,
                           "ms_median": med, "ms_min": ms[0], "bytes": byts,
                           "GBps": byts / med / 1e6, "frac_of_peak": byts / med / 1e6 / peak(),
                           "elements_per_s": n / med * 1e3, "plan": plan}), flush=True)
@@ -159,6 +178,7 @@ def main():
     ap.add_argument("case", nargs="+")
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--time", action="store_true")
+    ap.add_argument("--cold", action="store_true", help="flush L2 before every timed call")
     a = ap.parse_args()
     cache = {}
     for name in a.case:
@@ -169,7 +189,7 @@ def main():
             run_xform(name, a.reps, a.time)
             continue
         for c in cases(name):
-            run_reduce(*c, a.reps, a.time, cache)
+            run_reduce(*c, a.reps, a.time, cache, a.cold)
 
 
 if __name__ == "__main__":

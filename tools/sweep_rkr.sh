@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 OUT=gpurun_out/sweep_rkr_${TAG:-x}.jsonl
 : > $OUT
-CASES="cfg5-+-int32-gv cfg5-||-int32-gv cfg5-&&-fp32-gv cfg5-+-fp32-gv cfg5-+-int64-gv cfg5-&&-fp64-gv"
+CASES="cfg5-add-int32-gv cfg5-lor-int32-gv cfg5-land-fp32-gv cfg5-add-fp32-gv cfg5-add-int64-gv cfg5-land-fp64-gv"
 for c in $CASES; do
   XR_NO_RKR_STREAM=1 timeout 120 python tools/kdriver.py $c --reps 15 --time | sed 's/^{/{"variant": "seg", /' >> $OUT
   for s in auto 2 4 8 16 32; do
@@ -11,7 +11,7 @@ for c in $CASES; do
     env $E timeout 120 python tools/kdriver.py $c --reps 15 --time | sed "s/^{/{\"variant\": \"stream-$s\", /" >> $OUT
   done
 done
-for c in cfg5-+-int32-v cfg5-*-int32-v cfg5-&&-fp32-v; do
+for c in cfg5-add-int32-v cfg5-mul-int32-v cfg5-land-fp32-v; do
   for k in 2 4 8 16 32; do
     XR_ROWS_UNITS_PER_CTA=$k timeout 120 python tools/kdriver.py $c --reps 15 --time | sed "s/^{/{\"variant\": \"rows-k$k\", /" >> $OUT
   done
