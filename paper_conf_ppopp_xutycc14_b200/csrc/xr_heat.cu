@@ -135,8 +135,7 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
   const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
   if (threadIdx.x == 0) {
     a.partials[cta] = err;
-    __threadfence();
-    const unsigned t = atomicAdd(a.tickets, 1u);
+    const unsigned t = ticket_add(a.tickets);
     s_last = (t == (unsigned)(a.ntiles - 1));
   }
   __syncthreads();
@@ -247,8 +246,7 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
   const int64_t cta = (int64_t)blockIdx.y * gridDim.x + blockIdx.x;
   if (tid == 0) {
     a.partials[cta] = err;
-    __threadfence();
-    const unsigned t = atomicAdd(a.tickets, 1u);
+    const unsigned t = ticket_add(a.tickets);
     s_last = (t == (unsigned)(a.ntiles - 1));
   }
   cons_sync();
@@ -308,7 +306,7 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
     if (lane == 0) {
       int64_t q = 0;  // global row counter (slot = q % kHeatSlots)
       int seq = 0;
-      long long t = claim_first();
+      long long t = claim_first(pa.sched);
       while (true) {
         const long long nt = claim_next(pa.sched);
         const int slot0 = (int)(q % kHeatSlots);
@@ -394,8 +392,7 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
   err = cons_reduce<OP_MAX, double>(err, smem, cw, lane);
   if (tid == 0) {
     a.partials[blockIdx.x] = err;
-    __threadfence();
-    s_last = (atomicAdd(a.tickets, 1u) == gridDim.x - 1u);
+    s_last = (ticket_add(a.tickets) == gridDim.x - 1u);
   }
   cons_sync();
   if (s_last) {

@@ -270,7 +270,7 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
 
   if constexpr (W == BLOCK) {
     __shared__ long long s_unit[2];
-    if (threadIdx.x == 0) s_unit[0] = claim_first();
+    if (threadIdx.x == 0) s_unit[0] = claim_first(a.sched);
     __syncthreads();
     long long u = s_unit[0];
     int par = 1;
@@ -288,8 +288,7 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
       } else {  // a4: gang tier, last CTA of output o combines its S partials
         if (threadIdx.x == 0) {
           partials[u] = v;
-          __threadfence();
-          const unsigned t = atomicAdd(&a.tickets[o], 1u);
+          const unsigned t = ticket_add(&a.tickets[o]);
           s_last = (t == (unsigned)(S - 1));
         }
         __syncthreads();
@@ -329,8 +328,7 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
         int last = 0;
         if (lane == 0) {
           partials[u] = v;
-          __threadfence();
-          const unsigned t = atomicAdd(&a.tickets[o], 1u);
+          const unsigned t = ticket_add(&a.tickets[o]);
           last = (t == (unsigned)(S - 1));
         }
         last = __shfl_sync(0xffffffffu, last, 0);
@@ -432,7 +430,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = claim_first();
+      long long u = claim_first(a.sched);
       while (true) {
         const long long nu = claim_next(a.sched);  // next claim, in flight
         const int slot0 = (int)(g % NS);
@@ -525,8 +523,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
     } else {
       if (ct == 0) {
         partials[u] = v;
-        __threadfence();
-        const unsigned t = atomicAdd(&a.tickets[o], 1u);
+        const unsigned t = ticket_add(&a.tickets[o]);
         s_last = (t == (unsigned)(S - 1));
       }
       cons_sync();
@@ -545,8 +542,7 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
   }
   if (whole) {  // a4: one ticket per CTA; the last CTA folds the S unit partials in unit order
     if (ct == 0) {
-      __threadfence();
-      const unsigned t = atomicAdd(&a.tickets[0], 1u);
+      const unsigned t = ticket_add(&a.tickets[0]);
       s_last = (t == gridDim.x - 1u);
     }
     cons_sync();
@@ -607,7 +603,7 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = claim_first();
+      long long u = claim_first(a.sched);
       while (true) {
         const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
@@ -813,8 +809,7 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
       for (int c = t; c < a.K; c += kBlock) P1[s * a.K + c] = col[c];
       __syncthreads();
       if (t == 0) {
-        __threadfence();
-        s_last = (atomicAdd(&gt[gi], 1u) == (unsigned)(gsz - 1));
+        s_last = (ticket_add(&gt[gi]) == (unsigned)(gsz - 1));
       }
       __syncthreads();
       if (s_last) {
@@ -828,8 +823,7 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
           __syncthreads();
           if (t == 0) {
             gt[gi] = 0u;
-            __threadfence();
-            s_last = (atomicAdd(tt, 1u) == (unsigned)(a.G2 - 1));
+            s_last = (ticket_add(tt) == (unsigned)(a.G2 - 1));
           }
           __syncthreads();
           if (s_last) {
@@ -859,6 +853,22 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
 // the last unit of output j folds its S partials.  (A first version streamed
 // all rows and folded them by j into K-wide shared-memory partial rows: 0.60
 // of peak, latency bound on the partial-row folds, r01.)
+// Unit u -> (j-block, k split).  k-split-major (XR_RKR_KMAJOR=1): units that
+// run at the same time read different j-blocks, i.e. different 16 KiB offsets
+// within the 1 MiB k stride, instead of the same offset of many k planes.
+#ifndef XR_RKR_KMAJOR
+#define XR_RKR_KMAJOR 1
+#endif
+__device__ __forceinline__ void rkr_unit(int64_t u, int64_t S, int64_t njb, int64_t* jb, int64_t* s) {
+#if XR_RKR_KMAJOR
+  *s = u / njb;
+  *jb = u - *s * njb;
+#else
+  *jb = u / S;
+  *s = u - *jb * S;
+#endif
+}
+
 template <int OP, typename T, int NS>
 __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ RkrArgs a) {
   using O = Op<OP, T>;
@@ -891,7 +901,7 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = claim_first();
+      long long u = claim_first(a.sched);
       while (true) {
         const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
@@ -902,7 +912,8 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
           mbar_arrive(&full[slot0]);
           break;
         }
-        const int64_t jb = u / S, s = u - jb * S;
+        int64_t jb, s;
+        rkr_unit(u, S, a.units / S, &jb, &s);
         const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
         const unsigned nb = (unsigned)(min((int64_t)J, a.K - jb * J) << rshift);
         const char* src = static_cast<const char*>(a.in) + ((k0 * a.K + jb * J) << rshift);
@@ -931,7 +942,8 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
     mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
-    const int64_t jb = u / S, s = u - jb * S;
+    int64_t jb, s;
+        rkr_unit(u, S, a.units / S, &jb, &s);
     const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
     const int nrows = (int)min((int64_t)J, a.K - jb * J);
     Acc acc[4][VEC];
@@ -976,8 +988,7 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
           int last = 0;
           if (lane == 0) {
             partials[o * S + s] = v;
-            __threadfence();
-            last = (atomicAdd(&a.tickets[o], 1u) == (unsigned)(S - 1));
+            last = (ticket_add(&a.tickets[o]) == (unsigned)(S - 1));
           }
           last = __shfl_sync(0xffffffffu, last, 0);
           if (last) {
@@ -1020,7 +1031,7 @@ __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_co
   const int64_t per_b = a.tiles * a.S;
 
   __shared__ long long s_unit[2];
-  if (t == 0) s_unit[0] = claim_first();
+  if (t == 0) s_unit[0] = claim_first(a.sched);
   __syncthreads();
   long long u = s_unit[0];
   int par = 1;
@@ -1085,8 +1096,7 @@ __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_co
       if (t < TW) P[s * TW + t] = v;
       __syncthreads();  // the CTA's partial stores happen-before thread 0's fence (cumulative)
       if (t == 0) {
-        __threadfence();
-        const unsigned tk = atomicAdd(&a.tickets[b * a.tiles + tile], 1u);
+        const unsigned tk = ticket_add(&a.tickets[b * a.tiles + tile]);
         s_last = (tk == (unsigned)(a.S - 1));
       }
       __syncthreads();
@@ -1179,7 +1189,7 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
     if (lane == 0) {
       int64_t g = 0;
       int seq = 0;
-      long long u = claim_first();
+      long long u = claim_first(a.sched);
       while (true) {
         const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
@@ -1303,8 +1313,7 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
       if (tid < TW) P1[s * TW + tid] = v;
       cons_sync();  // partial stores happen-before thread 0's (cumulative) fence
       if (tid == 0) {
-        __threadfence();
-        const unsigned tk = atomicAdd(&gt[grp_i], 1u);
+        const unsigned tk = ticket_add(&gt[grp_i]);
         s_last = (tk == (unsigned)(gsz - 1));
       }
       cons_sync();
@@ -1318,8 +1327,7 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
           if (tid < TW) P2[grp_i * TW + tid] = w;
           cons_sync();
           if (tid == 0) {
-            __threadfence();
-            const unsigned tk = atomicAdd(tt, 1u);
+            const unsigned tk = ticket_add(tt);
             s_last = (tk == (unsigned)(a.G2 - 1));
           }
           cons_sync();

@@ -139,12 +139,40 @@ namespace xr {
 // Dynamic unit claiming for CTA-wide work: thread 0 fetches the next unit
 // index (prefetched one unit ahead into a parity slot) from a device counter;
 // the last CTA to exit resets the counters for the next launch.
-// The first unit of every CTA is static (blockIdx.x): the first dynamic claim
-// would put an L2 atomic round trip before the first load of every CTA.
-__device__ __forceinline__ long long claim_first() { return (long long)blockIdx.x; }
+// Gang-tier ticket (a4): __threadfence() orders the partial(s) written before
+// it (cumulatively: the CTA's writes ordered before by bar.sync) ahead of the
+// increment; the last arriver fences again before reading the partials.
+// XR_TICKET_ACQREL=1: one atom.add.acq_rel.gpu instead (measured neutral, r01
+// A/B; the proven fence + atomic stays the default)
+#ifndef XR_TICKET_ACQREL
+#define XR_TICKET_ACQREL 0
+#endif
+__device__ __forceinline__ unsigned ticket_add(unsigned* t) {
+#if XR_TICKET_ACQREL
+  unsigned v;
+  asm volatile("atom.add.acq_rel.gpu.global.u32 %0, [%1], 1;" : "=r"(v) : "l"(t) : "memory");
+  return v;
+#else
+  __threadfence();
+  return atomicAdd(t, 1u);
+#endif
+}
+
+// XR_STATIC_FIRST=1: every CTA's first unit is blockIdx.x (saves one claim
+// round trip) -- measured neutral on streams and 8% SLOWER on 512^3 32-bit GW
+// columns (r01 A/B), so the first unit is claimed like the others.
+#ifndef XR_STATIC_FIRST
+#define XR_STATIC_FIRST 0
+#endif
+#if XR_STATIC_FIRST
+__device__ __forceinline__ long long claim_first(unsigned long long*) { return (long long)blockIdx.x; }
 __device__ __forceinline__ long long claim_next(unsigned long long* c) {
   return (long long)gridDim.x + (long long)atomicAdd(c, 1ull);
 }
+#else
+__device__ __forceinline__ long long claim_next(unsigned long long* c) { return (long long)atomicAdd(c, 1ull); }
+__device__ __forceinline__ long long claim_first(unsigned long long* c) { return claim_next(c); }
+#endif
 __device__ __forceinline__ void sched_exit(unsigned long long* c) {
   if (threadIdx.x == 0) {
     __threadfence();

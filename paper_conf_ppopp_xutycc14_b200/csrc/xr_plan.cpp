@@ -12,8 +12,11 @@
 //      no-op), (2) merge adjacent levels of the same status (row-major
 //      adjacent levels are one contiguous level), (3) the remaining pattern is
 //      one of R, KR, RK, KRK, RKR, K.
+#include <unistd.h>  // environ
+
 #include <algorithm>
 #include <cstdlib>
+#include <cstring>
 
 #include "../../include/xreduce.h"
 #include "xr_internal.h"
@@ -29,6 +32,26 @@ int acc_size(int op, int dtype) {
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+// Tuning / A-B overrides (XR_*), read on every call so tests can flip them,
+// but with ONE pass over the environment instead of a getenv scan per name
+// (the planner runs on every launch; r01: ~1 us of host time per call).
+namespace {
+struct XrEnv {
+  int n = 0;
+  const char* kv[16];
+  const char* get(const char* name) const {
+    const size_t len = std::strlen(name);
+    for (int i = 0; i < n; ++i)
+      if (std::strncmp(kv[i], name, len) == 0 && kv[i][len] == '=') return kv[i] + len + 1;
+    return nullptr;
+  }
+};
+void scan_env(XrEnv* e) {
+  for (char** p = environ; p && *p && e->n < 16; ++p)
+    if ((*p)[0] == 'X' && (*p)[1] == 'R' && (*p)[2] == '_') e->kv[e->n++] = *p;
+}
+}  // namespace
+
 int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
   int64_t cap = (int64_t)std::max(num_sms, 1) * std::max(ctas_per_sm, 1);
   return std::max<int64_t>(1, std::min(units, cap));
@@ -37,6 +60,8 @@ int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
                int num_sms, Plan* p, bool seg_only) {
   *p = Plan();
+  XrEnv env;
+  scan_env(&env);
   bool seg_only_small = false;
   const int size = dtype_size(dtype);
   const int vec = 16 / size;
@@ -88,8 +113,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   {
     int64_t total = 1;
     for (int d = 0; d < 3; ++d) total *= dims[d];
-    const char* env = std::getenv("XR_SMALL_BYTES");  // test / tuning override
-    const int64_t small = env ? std::atoll(env) : kSmallBytes;
+    const char* sb = env.get("XR_SMALL_BYTES");  // test / tuning override
+    const int64_t small = sb ? std::atoll(sb) : kSmallBytes;
     if (total * size < small) seg_only_small = true;
   }
 
@@ -120,11 +145,11 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int64_t row_bytes = K * size;
     const bool pow2 = (row_bytes & (row_bytes - 1)) == 0;
     if (aligned && pow2 && row_bytes >= 16 &&
-        (row_bytes <= 512 || (seg_only_small && row_bytes <= 4096)) && std::getenv("XR_NO_FLAT") == nullptr) {
+        (row_bytes <= 512 || (seg_only_small && row_bytes <= 4096)) && env.get("XR_NO_FLAT") == nullptr) {
       const int64_t rp4k = 4096 / row_bytes;
       const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch
-      const char* eu = std::getenv("XR_FLAT_UNITS_PER_CTA");  // tuning overrides
-      const char* er = std::getenv("XR_FLAT_MIN_ROUNDS");
+      const char* eu = env.get("XR_FLAT_UNITS_PER_CTA");  // tuning overrides
+      const char* er = env.get("XR_FLAT_MIN_ROUNDS");
       // ~1 long unit per resident CTA: each unit's epilogue folds a K-wide
       // partial row, so long units win (r01 sweep: 256 units 4.7 TB/s, 4096
       // units 2.5 TB/s on the paper's 2^20 x 2 x 32 int32 gang case)
@@ -150,7 +175,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
     if (!seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
-        B < (int64_t(1) << 31) && std::getenv("XR_NO_TMA") == nullptr) {
+        B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr) {
       const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
       const int64_t tiles = cdiv(K, TWt);
       // Balance (measured r01 sweeps): the producer warp keeps every CTA's ring
@@ -159,7 +184,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       // stragglers for a third round).  k units per CTA, grid = units / k.
       const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;  // resident CTAs (64 KiB ring each)
       const int64_t base = B * tiles;
-      const char* upc = std::getenv("XR_COLTMA_UNITS_PER_CTA");  // tuning override
+      const char* upc = env.get("XR_COLTMA_UNITS_PER_CTA");  // tuning override
       // measured (r01 sweeps): 2 units per CTA is best with few column tiles
       // (512^3 G/W/GW: 0.95/0.95/0.97 at 1 GiB); with many tiles (cfg3: 128)
       // ~512 KiB units (up to 16 per CTA) win (1.04 vs 1.02)
@@ -234,13 +259,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // bulk copy of J contiguous rows, accumulated per warp in registers.
   if (!seg_only && !seg_only_small && nr == 3 && row_bytes >= 512 && row_bytes <= 2048 &&
       (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= kStageBytes / row_bytes &&
-      std::getenv("XR_NO_RKR") == nullptr && std::getenv("XR_NO_BULK") == nullptr) {
+      env.get("XR_NO_RKR") == nullptr && env.get("XR_NO_BULK") == nullptr) {
     const int64_t J = kStageBytes / row_bytes;
     const int64_t njb = cdiv(O, J);
     const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;  // resident CTAs (64 KiB ring each)
-    const char* eu = std::getenv("XR_RKR_UNITS_PER_CTA");   // tuning override
-    // r01 sweep (512^3 32-bit GV): 4 units per CTA 0.89, 8 0.91, 16 0.81, 32 0.82
-    const int64_t k = eu ? std::max(1, std::atoi(eu)) : 8;
+    const char* eu = env.get("XR_RKR_UNITS_PER_CTA");   // tuning override
+    // r01 sweeps (512^3 32-bit GV): 4-6 units per CTA 0.89, 8 0.87-0.91, 12 0.87, 16 0.81
+    const int64_t k = eu ? std::max(1, std::atoi(eu)) : 4;
     // k units per resident CTA, each >= kStages stages (k values)
     int64_t S = std::max<int64_t>(1, std::min<int64_t>(cdiv(k * cap, njb), C / kStages));
     // fp32 '+': each lane accumulator folds vpl elements per k (chains <= kChainCap)
@@ -265,7 +290,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
   if (!seg_only && !seg_only_small && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 &&
       (row_bytes & (row_bytes - 1)) == 0 &&
-      in_addr % 16 == 0 && std::getenv("XR_NO_BULK") == nullptr) {
+      in_addr % 16 == 0 && env.get("XR_NO_BULK") == nullptr) {
     const int64_t rps = kStageBytes / row_bytes;
     const int64_t nst = cdiv(O, rps);
     const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;
@@ -273,7 +298,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     // epilogue, the producer streams across it), and short units balance the
     // tail (r01 sweep, 512^3 32-bit V: 2 units per CTA 0.91 of peak, 8 0.95,
     // 32 1.00)
-    const char* eu = std::getenv("XR_ROWS_UNITS_PER_CTA");  // tuning override
+    const char* eu = env.get("XR_ROWS_UNITS_PER_CTA");  // tuning override
     const int64_t k = eu ? std::max(1, std::atoi(eu)) : 32;
     const int64_t units = std::max<int64_t>(1, std::min<int64_t>(nst, k * cap));
     p->kernel = K_ROWS;
@@ -308,10 +333,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // unit's rows (one bulk copy per row piece).  r01 sweep on 512^3 GV: 64-bit
   // (4 KiB rows) 0.95-1.01 of peak vs 0.66-0.95 for the seg kernel; 32-bit
   // (2 KiB rows) no better than seg (0.83-0.87 both), so those stay on seg.
-  const char* rkr_min = std::getenv("XR_RKR_STREAM_MIN_ROW");  // tuning override (bytes)
+  const char* rkr_min = env.get("XR_RKR_STREAM_MIN_ROW");  // tuning override (bytes)
   const bool rkr_stream = nr == 3 && row_bytes >= (rkr_min ? std::atoll(rkr_min) : 4096) &&
-                          row_bytes % 16 == 0 && in_addr % 16 == 0 && std::getenv("XR_NO_RKR_STREAM") == nullptr;
-  const bool stream = !seg_only && !seg_only_small && std::getenv("XR_NO_BULK") == nullptr &&
+                          row_bytes % 16 == 0 && in_addr % 16 == 0 && env.get("XR_NO_RKR_STREAM") == nullptr;
+  const bool stream = !seg_only && !seg_only_small && env.get("XR_NO_BULK") == nullptr &&
                       ((C == 1 && row_bytes >= (int64_t)kStages * kStageBytes) || rkr_stream);
   if (stream) {
     // several outputs: amortise the epilogue (RKR: 512 KiB units, r01 sweep)
@@ -320,8 +345,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   }
   // fp32 '+': per-thread chains <= kChainCap (stream: 16 accumulators per thread)
   if (chain_capped) S = std::max<int64_t>(S, cdiv(work, (int64_t)kChainCap * W * vec * kUnroll));
-  if (stream && std::getenv("XR_STREAM_SPLITS") != nullptr)  // tuning override
-    S = std::max<int64_t>(1, std::atoll(std::getenv("XR_STREAM_SPLITS")));
+  if (stream && env.get("XR_STREAM_SPLITS") != nullptr)  // tuning override
+    S = std::max<int64_t>(1, std::atoll(env.get("XR_STREAM_SPLITS")));
   if (stream) W = kBlock;  // CTA-wide units, claimed dynamically
   if (S > 1 && W < 32) W = 32;  // the gang-tier ticket runs per warp or per CTA
   int64_t Sr, Sc;

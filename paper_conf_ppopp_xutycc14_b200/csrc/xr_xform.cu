@@ -164,8 +164,7 @@ __global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in
     } else {
       if (threadIdx.x == 0) {
         partials[u] = v;
-        __threadfence();
-        s_last = (atomicAdd(&a.tickets[o], 1u) == (unsigned)(S - 1));
+        s_last = (ticket_add(&a.tickets[o]) == (unsigned)(S - 1));
       }
       __syncthreads();
       if (s_last) {
