@@ -133,9 +133,10 @@ int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level
  *               XR_ERR_UNSUPPORTED), no FMA (@35389).  out is int64.
  *   XR_XF_DOT   inner product, Fig 13(b) (@41386-42177): out[o] = init +
  *               sum x*y in dtype (ints wrap, C6; fp within the C9 bound).
- * level_mask as xr_reduce.  Canonical shapes R, KR, RKR and K are supported;
- * column shapes (RK, KRK: the reduced levels are all outside a kept
- * contiguous level) return XR_ERR_UNSUPPORTED.  One launch, single pass. */
+ * level_mask as xr_reduce; every canonical shape (R, KR, RK, KRK, RKR, K) is
+ * supported.  Column shapes (the reduced levels all outside a kept contiguous
+ * level) read 16-B vectors of both inputs when both are 16-B aligned and the
+ * kept row is a multiple of 16 B, else scalars.  One launch, single pass. */
 typedef enum { XR_XF_DISK = 1, XR_XF_DOT = 2 } xr_xform;
 int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                         const void* x, const void* y, void* out, xr_stream_t stream);
@@ -147,8 +148,12 @@ int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims[3], unsign
  * (DEVICE, xr_out_count elements); all share nest_dims and level_mask (with
  * XR_INIT_FROM_OUT applying to every output).  1 <= nvars <= 8.  Semantics per
  * variable exactly as xr_reduce; no output may overlap an input or another
- * output.  Canonical shapes R, KR, RKR, K and empty reduced extents are
- * supported; column shapes (RK, KRK) return XR_ERR_UNSUPPORTED.  One launch. */
+ * output.  Every canonical shape (R, KR, RK, KRK, RKR, K) and empty extents
+ * are supported.  One launch (none if every output is empty).
+ * Errors (nothing is launched): XR_ERR_INVALID for nvars outside [1, 8], a
+ * bad op / dtype / mask, a null or misaligned pointer with non-empty work, or
+ * overlapping buffers; XR_ERR_UNSUPPORTED for & | ^ on fp; XR_ERR_CUDA if the
+ * launch fails. */
 typedef struct {
   int op;          /* xr_op   */
   int dtype;       /* xr_dtype */
@@ -157,6 +162,26 @@ typedef struct {
 } xr_var;
 int xr_reduce_multi(int nvars, const xr_var* vars, const int64_t nest_dims[3], unsigned level_mask,
                     xr_stream_t stream);
+
+/* Different variables reduced at DIFFERENT levels of one nest, in one launch
+ * (PAPER.md 3.2 @27198-27253: "reduction can also occur on different
+ * variables within different levels of parallelism", e.g. i_sum at the vector
+ * level and j_sum at the worker level of the same nest).
+ * As xr_reduce_multi, but each variable carries its own level_mask (any legal
+ * xr_reduce mask, XR_INIT_FROM_OUT per variable) and its output holds
+ * xr_out_count(nest_dims, level_mask) elements of its dtype.  Each variable's
+ * result is exactly xr_reduce(op, dtype, nest_dims, level_mask, in, out).
+ * Variables may share an input (e.g. row sums and the total of one array);
+ * outputs may not overlap any input or another output.  Errors as
+ * xr_reduce_multi.  One launch. */
+typedef struct {
+  int op;               /* xr_op    */
+  int dtype;            /* xr_dtype */
+  unsigned level_mask;  /* XR_GANG | XR_WORKER | XR_VECTOR [| XR_INIT_FROM_OUT] */
+  const void* in;
+  void* out;
+} xr_var_at;
+int xr_reduce_multi_at(int nvars, const xr_var_at* vars, const int64_t nest_dims[3], xr_stream_t stream);
 
 /* The paper's own code-generation scheme, an in-house A/B
  * baseline on the same GPU: Kepler-style launch of num_gangs blocks of

@@ -65,6 +65,11 @@ class Var(ctypes.Structure):
                 ("out", ctypes.c_void_p)]
 
 
+class VarAt(ctypes.Structure):
+    _fields_ = [("op", ctypes.c_int), ("dtype", ctypes.c_int), ("level_mask", ctypes.c_uint),
+                ("in_", ctypes.c_void_p), ("out", ctypes.c_void_p)]
+
+
 class ShardInfo(ctypes.Structure):
     _fields_ = [("collective", ctypes.c_int), ("nccl_op", ctypes.c_int),
                 ("merge_init", ctypes.c_int), ("local_init_from_out", ctypes.c_int),
@@ -103,6 +108,7 @@ _SIGS = {
     "xr_transform_reduce": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_paper": (_c, [_c, _c, _i64p, _u, _vp, _vp, _c, _c, _c, _vp]),
     "xr_reduce_multi": (_c, [_c, ctypes.POINTER(Var), _i64p, _u, _vp]),
+    "xr_reduce_multi_at": (_c, [_c, ctypes.POINTER(VarAt), _i64p, _vp]),
     "xr_heat_step_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp, _vp]),
     "xr_heat_run_sharded_sim": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _c, ctypes.POINTER(_vp),
@@ -220,6 +226,14 @@ def xr_reduce_multi(variables, nest_dims, level_mask, stream: int = 0) -> int:
     vs = list(variables)
     arr = (Var * len(vs))(*[Var(_op(o), _dt(d), i or None, p or None) for o, d, i, p in vs])
     return _lib.xr_reduce_multi(len(vs), arr, _dims(nest_dims), mask_of(level_mask), stream or None)
+
+
+def xr_reduce_multi_at(variables, nest_dims, stream: int = 0) -> int:
+    """variables: iterable of (op, dtype, level_mask, in_ptr, out_ptr) -- each
+    variable reduced at its own levels, one launch (include/xreduce.h)."""
+    vs = list(variables)
+    arr = (VarAt * len(vs))(*[VarAt(_op(o), _dt(d), mask_of(m), i or None, p or None) for o, d, m, i, p in vs])
+    return _lib.xr_reduce_multi_at(len(vs), arr, _dims(nest_dims), stream or None)
 
 
 def xr_reduce_paper(op, dtype, nest_dims, level_mask, in_ptr: int, out_ptr: int, num_gangs: int = 0,

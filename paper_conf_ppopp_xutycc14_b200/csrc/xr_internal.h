@@ -111,10 +111,15 @@ struct Plan {
 
 // Pure host: validation happens before (api.cpp).  in_addr only matters for
 // its alignment (16-B vector path of the column kernel).
-// seg_only: plan for the register seg decomposition only, with CTA-wide
-// groups (no stream / rows / TMA kernels) -- used by the transform-reduce.
+// seg_only: plan for the register seg / column decompositions only, with
+// CTA-wide groups (no stream / rows / TMA kernels) -- used by the fused
+// transform-reduce and multi-variable launches.  want_units (> 0, seg_only
+// only): the number of work units to aim for instead of the default
+// over-decomposition (the multi-variable launch shares one grid among its
+// variables), counted in CTA-wide units.  sub_cta (seg_only only): short rows
+// keep the sub-CTA groups of 8 / 32 lanes (p->group) instead of CTA-wide ones.
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p, bool seg_only = false);
+               int num_sms, Plan* p, bool seg_only = false, int64_t want_units = 0, bool sub_cta = false);
 
 int dtype_size(int dtype);
 int acc_size(int op, int dtype);

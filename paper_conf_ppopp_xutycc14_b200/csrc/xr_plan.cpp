@@ -58,7 +58,7 @@ int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
 }
 
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p, bool seg_only) {
+               int num_sms, Plan* p, bool seg_only, int64_t want_override, bool sub_cta) {
   *p = Plan();
   XrEnv env;
   scan_env(&env);
@@ -136,15 +136,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     else { B = run_n[0]; R = run_n[1]; K = run_n[2]; p->shape = XR_SHAPE_KRK; }
     const bool aligned = ((K * size) % 16 == 0) && (in_addr % 16 == 0);
     const int cv = aligned ? vec : 1;
-    if (seg_only) {
-      p->kernel = K_COL;
-      return;
-    }
+    // seg_only (the fused multi-input / multi-variable launches): always the
+    // register column decomposition below (their col_unit, xr_colunit.cuh)
     // Narrow rows (power-of-two row_bytes in [16, 512] B, or up to 4 KiB for
     // small inputs): the flat column kernel streams whole rows contiguously.
     const int64_t row_bytes = K * size;
     const bool pow2 = (row_bytes & (row_bytes - 1)) == 0;
-    if (aligned && pow2 && row_bytes >= 16 &&
+    if (!seg_only && aligned && pow2 && row_bytes >= 16 &&
         (row_bytes <= 512 || (seg_only_small && row_bytes <= 4096)) && env.get("XR_NO_FLAT") == nullptr) {
       const int64_t rp4k = 4096 / row_bytes;
       const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch
@@ -174,7 +172,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       return;
     }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
-    if (!seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
+    if (!seg_only && !seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr) {
       const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
       const int64_t tiles = cdiv(K, TWt);
@@ -222,8 +220,9 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int64_t NW = kBlock / 32;
     int64_t S = 1;
     const int64_t base = B * tiles;
-    if (base < kUnitsPerCta * target_ctas) {
-      S = cdiv(kUnitsPerCta * target_ctas, base);
+    const int64_t want_col = (seg_only && want_override > 0) ? want_override : kUnitsPerCta * target_ctas;
+    if (base < want_col) {
+      S = cdiv(want_col, base);
       // >= 4 load rounds per warp: on small inputs a split's extra ticket round
       // costs more than its parallelism buys (cfg1 G/W: 4.0 us unsplit vs 5.4 us)
       S = std::min<int64_t>(S, std::max<int64_t>(1, R / (4 * NW * kUnroll)));
@@ -313,12 +312,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     s.Sr = 1; s.Sc = units; s.units = units;
     return;
   }
-  int W = seg_only ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
+  int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
   const int64_t work = C * L;  // elements per output
   // CTA-wide groups claim units dynamically: over-decompose for tail balance
-  const int64_t want_units = (W == kBlock ? kUnitsPerCta : 2) * resident_groups(W);
+  const int64_t want_units = (seg_only && want_override > 0) ? want_override * (kBlock / W)
+                             : (W == kBlock ? kUnitsPerCta : 2) * resident_groups(W);
   int64_t S = 1;
   if (O < want_units) {
     S = cdiv(want_units, O);

@@ -7,14 +7,16 @@
 //   XR_XF_DOT: inner product (Fig 13(b) @41386-42177): sum of x*y, dtype out.
 // Single pass like xr_reduce: private partials (16-B loads of BOTH inputs,
 // 4+4 in flight), warp shuffles, CTA smem combine, last-CTA ticket.
-// Canonical shapes R, KR, RKR (the seg decomposition) and K; column shapes
-// (RK, KRK) return XR_ERR_UNSUPPORTED.
+// Canonical shapes R, KR, RKR (the seg decomposition), K, and the column
+// shapes RK, KRK (xr_colunit.cuh: lanes own contiguous kept columns of BOTH
+// inputs, warps stride the reduced rows, per-tile ticket).
 #include <algorithm>
 #include <cstdlib>
 
 #include "../../include/xreduce.h"
 #include "xr_internal.h"
 #include "xr_ops.cuh"
+#include "xr_colunit.cuh"
 
 namespace xr {
 
@@ -196,6 +198,28 @@ __global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const vo
   }
 }
 
+// Column shapes (RK, KRK): CTA-wide column units, static round robin.
+template <int XF, typename T, int VEC>
+__global__ void __launch_bounds__(kBlock) xform_col_kernel(const __grid_constant__ ColArgs a, const void* in2) {
+  using X = Xf<XF, T>;
+  __shared__ __align__(16) unsigned char sm[col_unit_smem<X, VEC>()];
+  __shared__ int s_last;
+  for (int64_t u = blockIdx.x; u < a.units; u += gridDim.x)
+    col_unit<X, T, 2, VEC, kUnroll>(a, static_cast<const T*>(a.in), static_cast<const T*>(in2), u, sm, &s_last);
+}
+
+template <int XF, typename T, int VEC>
+static void xform_col_launch(const ColArgs& c, const void* in2, int sms, cudaStream_t s) {
+  static int occ = [] {
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xform_col_kernel<XF, T, VEC>, kBlock, 0) != cudaSuccess ||
+        n < 1)
+      n = 1;
+    return n;
+  }();
+  xform_col_kernel<XF, T, VEC><<<(unsigned)grid_for(c.units, sms, occ), kBlock, 0, s>>>(c, in2);
+}
+
 template <int XF, typename T>
 static cudaError_t xform_launch(Plan& p, const void* in2, int sms, cudaStream_t s) {
   if (p.kernel == K_FILL || p.kernel == K_IDENT) {
@@ -203,6 +227,9 @@ static cudaError_t xform_launch(Plan& p, const void* in2, int sms, cudaStream_t 
     if (p.kernel == K_FILL) e.in = nullptr;
     const int64_t grid = grid_for((e.n + kBlock - 1) / kBlock, sms, 8);
     xform_ident_kernel<XF, T><<<(unsigned)grid, kBlock, 0, s>>>(e, in2);
+  } else if (p.kernel == K_COL) {
+    if (p.vec > 1) xform_col_launch<XF, T, 16 / sizeof(T)>(p.col, in2, sms, s);
+    else xform_col_launch<XF, T, 1>(p.col, in2, sms, s);
   } else {
     static int occ = [] {
       int n = 0;
@@ -242,18 +269,20 @@ extern "C" int xr_transform_reduce(int xform, int dtype, const int64_t nest_dims
   if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  // in_addr: the column path takes 16-B vectors only if BOTH inputs are aligned
   make_plan(xform == XR_XF_DOT ? XR_OP_ADD : XR_OP_LOR /* non-chain-capped */, dtype, nest_dims, level_mask & 7u,
-            0, sms, &p, /*seg_only=*/true);
+            (uint64_t)((uintptr_t)x | (uintptr_t)y), sms, &p, /*seg_only=*/true);
   if (p.kernel == K_NONE) return XR_OK;
-  if (p.kernel == K_COL || p.kernel == K_COLTMA) return XR_ERR_UNSUPPORTED;
   // partial slots sized for the transform's accumulator (DISK: 8-byte counts)
-  const int64_t pbytes = p.splits > 1 ? p.units * 8 : 0;
+  const int64_t pslots = p.kernel == K_COL ? p.col.B * p.col.tiles * p.col.S * 32 * p.vec : p.units;
+  const int64_t pbytes = p.splits > 1 ? pslots * 8 : 0;
   void* partials = nullptr;
   unsigned* tickets = nullptr;
   int st = xform_workspace((cudaStream_t)stream, pbytes, p.tickets, &partials, &tickets);
   if (st) return st;
   const int ifo = (level_mask & XR_INIT_FROM_OUT) ? 1 : 0;
   p.seg.in = x; p.seg.out = out; p.seg.partials = partials; p.seg.tickets = tickets; p.seg.init_from_out = ifo;
+  p.col.in = x; p.col.out = out; p.col.partials = partials; p.col.tickets = tickets; p.col.init_from_out = ifo;
   p.elt.in = x; p.elt.out = out; p.elt.init_from_out = ifo;
   cudaStream_t s = (cudaStream_t)stream;
   cudaError_t e;

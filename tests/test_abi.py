@@ -91,6 +91,27 @@ def test_validation_without_gpu(xr):
     assert xr.xr_reduce_host("+", "int32", (0, 5, 5), 2, 0, 0) == xr.OK
 
 
+def test_multi_validation_without_gpu(xr):
+    """xr_reduce_multi / xr_reduce_multi_at validate every variable before any
+    CUDA call (include/xreduce.h): counts, masks, ops, alignment, overlaps."""
+    f = 0x100000
+    d = (2, 2, 2)
+    ok = ("+", "int32", "v", f, f * 4)
+    assert xr.xr_reduce_multi_at([], d) == xr.ERR_INVALID
+    assert xr.xr_reduce_multi_at([ok] * 9, d) == xr.ERR_INVALID
+    assert xr.xr_reduce_multi_at([ok, ("+", "int32", 0, f, f * 5)], d) == xr.ERR_INVALID        # no level
+    assert xr.xr_reduce_multi_at([ok, ("+", "int32", 0x11, f, f * 5)], d) == xr.ERR_INVALID     # stray bit
+    assert xr.xr_reduce_multi_at([ok, ("^", "fp64", "g", f, f * 5)], d) == xr.ERR_UNSUPPORTED
+    assert xr.xr_reduce_multi_at([ok, ("+", "fp64", "g", f, f * 5 + 4)], d) == xr.ERR_INVALID  # misaligned out
+    assert xr.xr_reduce_multi_at([ok, ("+", "fp64", "g", 0, f * 5)], d) == xr.ERR_INVALID      # null in
+    assert xr.xr_reduce_multi_at([ok, ("+", "int32", "gw", f, f * 4 + 8)], d) == xr.ERR_INVALID  # outputs overlap
+    assert xr.xr_reduce_multi_at([ok, ("+", "int32", "g", f * 4, f * 5)], d) == xr.ERR_INVALID  # out over an input
+    assert xr.xr_reduce_multi_at([ok], (-1, 2, 2)) == xr.ERR_INVALID
+    assert xr.xr_reduce_multi([("+", "int32", f, f * 4)] * 9, d, "g") == xr.ERR_INVALID
+    # every output empty: a valid no-op without any CUDA call
+    assert xr.xr_reduce_multi_at([("+", "int32", "g", 0, 0), ("max", "fp64", "gv", 0, 0)], (4, 0, 3)) == xr.OK
+
+
 # ------------------------------------------------------------------ planner (a0)
 SHAPE_TABLE = {
     # SURVEY.md 8(a) a0: mask -> canonical shape for a nest with 3 non-unit dims

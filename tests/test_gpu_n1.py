@@ -12,7 +12,8 @@ from gpu_util import TAU, torch_dt
 
 pytestmark = pytest.mark.gpu
 SEG_MASKS = ["v", "wv", "gv", "gwv"]   # canonical R / KR / RKR for 3 non-unit dims
-COL_MASKS = ["g", "w", "gw"]           # canonical RK / KRK -> unsupported
+COL_MASKS = ["g", "w", "gw"]           # canonical RK / KRK (column units, xr_colunit.cuh)
+ALL_MASKS = SEG_MASKS + COL_MASKS
 
 
 def run(xform, dtype, dims, levels, x, y, init=None, offset=0):
@@ -39,12 +40,14 @@ def run(xform, dtype, dims, levels, x, y, init=None, offset=0):
 
 
 @pytest.mark.parametrize("dtype", ["fp32", "fp64"])
-def test_disk_exact_counts_all_seg_masks(dtype):
-    for dims in [(7, 33, 129), (3, 5, 100003), (64, 64, 128)]:
+def test_disk_exact_counts_all_masks(dtype):
+    # ragged column widths (129: scalar column lanes; 128: 16-B column lanes;
+    # offset 1 misaligns both inputs), long reduced columns (5 x 70001 x 8)
+    for dims in [(7, 33, 129), (3, 5, 100003), (64, 64, 128), (5, 70001, 8), (9000, 3, 36)]:
         n = int(np.prod(dims))
         x = datagen.uniform_float(1, n, -1.0, 1.0, oracle.NP_DTYPES[dtype])
         y = datagen.uniform_float(2, n, -1.0, 1.0, oracle.NP_DTYPES[dtype])
-        for lv in SEG_MASKS:
+        for lv in ALL_MASKS:
             for off in (0, 1):
                 init = np.arange(oracle.out_count(dims, lv), dtype=np.int64) * 3
                 got = run("disk", dtype, dims, lv, x, y, init=init, offset=off)
@@ -66,9 +69,9 @@ def test_disk_lattice_and_boundary():
 
 
 @pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
-def test_dot_all_seg_masks(dtype):
+def test_dot_all_masks(dtype):
     dt = oracle.NP_DTYPES[dtype]
-    for dims in [(9, 17, 300), (2, 3, 70001), (40, 33, 65)]:
+    for dims in [(9, 17, 300), (2, 3, 70001), (40, 33, 65), (3, 40000, 12)]:
         n = int(np.prod(dims))
         if dtype.startswith("int"):
             x = datagen.uniform_int(3, n, -1000, 1000, dt)
@@ -76,23 +79,34 @@ def test_dot_all_seg_masks(dtype):
         else:
             x = datagen.uniform_float(3, n, -1.0, 1.0, dt)
             y = datagen.uniform_float(4, n, -1.0, 1.0, dt)
-        for lv in SEG_MASKS:
-            got = run("dot", dtype, dims, lv, x, y)
-            ref, S = oracle.transform_reduce("dot", dtype, dims, lv, x, y, want_abs=True)
-            if dtype.startswith("int"):
-                assert np.array_equal(got, ref)
-            else:
-                assert np.all(np.abs(got.astype(np.float64) - ref.astype(np.float64)) <= TAU[dtype] * S), lv
+        for lv in ALL_MASKS:
+            for off in (0, 1):
+                got = run("dot", dtype, dims, lv, x, y, offset=off)
+                ref, S = oracle.transform_reduce("dot", dtype, dims, lv, x, y, want_abs=True)
+                if dtype.startswith("int"):
+                    assert np.array_equal(got, ref), (dims, lv, off)
+                else:
+                    err = np.abs(got.astype(np.float64) - ref.astype(np.float64))
+                    assert np.all(err <= TAU[dtype] * S), (dims, lv, off)
 
 
-def test_unsupported_masks_and_dtypes():
+def test_dot_column_init_and_empty():
+    """Column shapes merge init once per output; an empty reduced extent gives out = init."""
+    x = datagen.uniform_int(5, 6 * 50 * 40, -50, 50, np.int64)
+    y = datagen.uniform_int(6, 6 * 50 * 40, -50, 50, np.int64)
+    for lv in COL_MASKS:
+        init = np.arange(oracle.out_count((6, 50, 40), lv), dtype=np.int64) - 7
+        got = run("dot", "int64", (6, 50, 40), lv, x, y, init=init)
+        assert np.array_equal(got, oracle.transform_reduce("dot", "int64", (6, 50, 40), lv, x, y, init=init))
+    init = np.arange(6 * 40, dtype=np.int64)
+    e = np.zeros(0, np.int64)
+    assert np.array_equal(run("dot", "int64", (6, 0, 40), "w", e, e, init=init), init)
+
+
+def test_unsupported_dtypes():
     import torch
     import paper_conf_ppopp_xutycc14_b200 as xr
-    x = torch.zeros(8 * 8 * 8, device="cuda")
     out = torch.zeros(64, device="cuda")
-    for lv in COL_MASKS:
-        assert xr.xr_transform_reduce("dot", "fp32", (8, 8, 8), lv, x.data_ptr(), x.data_ptr(),
-                                      out.data_ptr()) == xr.ERR_UNSUPPORTED
     xi = torch.zeros(8, dtype=torch.int32, device="cuda")
     assert xr.xr_transform_reduce("disk", "int32", (8, 1, 1), "g", xi.data_ptr(), xi.data_ptr(),
                                   out.data_ptr()) == xr.ERR_UNSUPPORTED

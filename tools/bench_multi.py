@@ -1,5 +1,6 @@
 #!/usr/bin/env python3
-"""N2 measurement: xr_reduce_multi (one launch) vs one xr_reduce per variable."""
+"""N2 measurement: xr_reduce_multi / xr_reduce_multi_at (one launch) vs one
+xr_reduce per variable; the A7b rows give every variable its own levels."""
 import json
 import os
 import sys
@@ -29,16 +30,23 @@ def timeit(fn, reps=21):
     return a.elapsed_time(b) / reps
 
 
-for dims, lv in [((64, 64, 128), "v"), ((64, 64, 128), "gwv"), ((4096, 1, 4096), "v"), ((1 << 24, 1, 1), "gwv")]:
+LEVELS_AT = ["v", "w", "g", "wv", "gw", "gv", "gwv", "w"]   # A7b: one mask per variable
+
+for dims, lv in [((64, 64, 128), "v"), ((64, 64, 128), "gwv"), ((4096, 1, 4096), "v"), ((1 << 24, 1, 1), "gwv"),
+                 ((64, 64, 128), "g"), ((1, 4096, 4096), "w"), ((64, 64, 128), "at"), ((256, 256, 256), "at")]:
     n = dims[0] * dims[1] * dims[2]
     xs = [(torch.rand(n, device="cuda") * 100).to(TDT[dt]) for _, dt in VARS]
-    cnt = xr.xr_out_count(dims, lv)
-    outs = [torch.zeros(cnt, dtype=TDT[dt], device="cuda") for _, dt in VARS]
+    lvs = LEVELS_AT if lv == "at" else [lv] * len(VARS)
+    outs = [torch.zeros(max(1, xr.xr_out_count(dims, m)), dtype=TDT[dt], device="cuda")
+            for (_, dt), m in zip(VARS, lvs)]
     sh = torch.cuda.current_stream().cuda_stream
-    spec = [(op, dt, x.data_ptr(), o.data_ptr()) for (op, dt), x, o in zip(VARS, xs, outs)]
-    t_multi = timeit(lambda: xr.xr_reduce_multi(spec, dims, lv, sh))
-    t_sep = timeit(lambda: [xr.xr_reduce(op, dt, dims, lv, i, o, sh) for op, dt, i, o in spec])
+    spec = [(op, dt, m, x.data_ptr(), o.data_ptr()) for (op, dt), m, x, o in zip(VARS, lvs, xs, outs)]
+    if lv == "at":
+        t_multi = timeit(lambda: xr.xr_reduce_multi_at(spec, dims, sh))
+    else:
+        t_multi = timeit(lambda: xr.xr_reduce_multi([(op, dt, i, o) for op, dt, _, i, o in spec], dims, lv, sh))
+    t_sep = timeit(lambda: [xr.xr_reduce(op, dt, dims, m, i, o, sh) for op, dt, m, i, o in spec])
     byts = sum(x.numel() * x.element_size() for x in xs)
-    print(json.dumps({"dims": dims, "levels": lv, "vars": len(VARS), "multi_ms": t_multi, "separate_ms": t_sep,
+    print(json.dumps({"dims": dims, "levels": lv if lv != "at" else lvs, "vars": len(VARS), "multi_ms": t_multi, "separate_ms": t_sep,
                       "speedup": t_sep / t_multi, "multi_GBps": byts / t_multi / 1e6,
                       "separate_GBps": byts / t_sep / 1e6}))
