@@ -189,10 +189,15 @@ int xr_reduce_multi_at(int nvars, const xr_var_at* vars, const int64_t nest_dims
  * 8), @35893-36486), Fig 3 loops, shared-memory interleaved log-step trees
  * (Figs 6c, 7, 8c) and, when the gang level reduces, a global partial buffer
  * plus a SECOND kernel launch (Fig 5c, @24887-25280; RMP @30925-31587).
- * Masks XR_GANG, XR_WORKER, XR_VECTOR and all three (the testsuite's single-
- * level and gang-worker-vector positions); ops + * max; dtypes int32, fp32,
- * fp64 (Table 2).  Other combinations: XR_ERR_UNSUPPORTED.  Same output
- * layout and init semantics as xr_reduce.  Two launches when gang reduces. */
+ * Masks XR_GANG, XR_WORKER, XR_VECTOR (the testsuite's single-level
+ * positions) and the three RMP scenarios of 3.2.1 (@28973-29561): gang &
+ * worker (global buffer of gangs x workers per output + second launch),
+ * worker & vector (shared-memory buffer of workers x vectors), gang & worker &
+ * vector (global buffer of every thread + second launch); gang & vector, which
+ * the paper says "cannot span ... without going through the worker", returns
+ * XR_ERR_UNSUPPORTED.  Ops + * max; dtypes int32, fp32, fp64 (Table 2).  Other
+ * combinations: XR_ERR_UNSUPPORTED.  Same output layout and init semantics as
+ * xr_reduce.  Two launches when gang reduces. */
 int xr_reduce_paper(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask, const void* in,
                     void* out, int num_gangs, int num_workers, int vector_length, xr_stream_t stream);
 

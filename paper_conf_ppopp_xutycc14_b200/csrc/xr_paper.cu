@@ -19,9 +19,12 @@
 // independent-thread-scheduling GPUs), and loops whose trip count differs
 // between threads of a block are padded so every thread reaches each
 // __syncthreads() (Fig 5a has a barrier inside while(j), a divergence hazard
-// when NJ % blockDim.y != 0).  Supported: masks g, w, v, gwv (Table 2's
-// single-level positions and RMP gwv), ops + * max, dtypes int32 fp32 fp64
-// (Table 2's Int / Float / Double).
+// when NJ % blockDim.y != 0).  Supported: masks g, w, v (Table 2's
+// single-level positions) and the paper's three RMP scenarios (3.2.1
+// @28973-29561: gang & worker, gang & worker & vector, worker & vector; gang &
+// vector "cannot span ... without going through the worker" and stays
+// unsupported), ops + * max, dtypes int32 fp32 fp64 (Table 2's Int / Float /
+// Double).
 #include <algorithm>
 
 #include "../../include/xreduce.h"
@@ -152,6 +155,55 @@ __global__ void paper_rmp_kernel(const T* in, typename Op<OP, T>::Acc* buf, int6
   buf[tid] = priv;
 }
 
+// ---- mask wv (RMP worker & vector, 3.2.1): the buffer of every reducing
+// thread (workers x vectors) lives in SHARED memory ("the buffer is stored in
+// the shared memory. Each thread writes its own partial reduction result into
+// this buffer and continues the reduction operation in the shared memory",
+// @28690-28973); one log-step over all of it per gang iteration k.
+template <int OP, typename T>
+__global__ void paper_wv_kernel(const T* in, T* out, int64_t NK, int64_t NJ, int64_t NI, int ifo) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  extern __shared__ unsigned char sraw[];
+  Acc* sbuf = reinterpret_cast<Acc*>(sraw);
+  const int tx = threadIdx.x, ty = threadIdx.y, bdx = blockDim.x, bdy = blockDim.y;
+  const int t = ty * bdx + tx, n = bdx * bdy;
+  for (int64_t k = blockIdx.x; k < NK; k += gridDim.x) {
+    Acc priv = O::identity();
+    for (int64_t j = ty; j < NJ; j += bdy)        // worker loop
+      for (int64_t i = tx; i < NI; i += bdx)      // vector loop
+        priv = O::combine(priv, O::lift(in[(k * NJ + j) * NI + i]));
+    sbuf[t] = priv;  // unique id of the thread
+    __syncthreads();
+    logstep<O>(sbuf, t, n, 1, true);
+    if (t == 0) {
+      const Acc init = ifo ? O::lift(out[k]) : O::identity();
+      out[k] = O::finish(O::combine(init, sbuf[0]));
+    }
+    __syncthreads();
+  }
+}
+
+// ---- mask gw (RMP gang & worker, 3.2.1), first launch: a GLOBAL buffer of
+// every reducing thread (gangs x workers) per kept vector iteration i ("the
+// buffer is allocated in the global memory since the reduction spans across
+// gangs", @29217-29414); layout [gang][worker][NI].  The second launch is
+// paper_second_kernel over rows = gangs * workers.
+template <int OP, typename T>
+__global__ void paper_gw_partial_kernel(const T* in, typename Op<OP, T>::Acc* buf, int64_t NK, int64_t NJ,
+                                        int64_t NI) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  const int64_t row = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
+  for (int64_t i = threadIdx.x; i < NI; i += blockDim.x) {  // vector loop (kept)
+    Acc priv = O::identity();
+    for (int64_t k = blockIdx.x; k < NK; k += gridDim.x)    // gang loop
+      for (int64_t j = threadIdx.y; j < NJ; j += blockDim.y)  // worker loop
+        priv = O::combine(priv, O::lift(in[(k * NJ + j) * NI + i]));
+    buf[row * NI + i] = priv;
+  }
+}
+
 template <int OP, typename T>
 static int paper_typed(const int64_t* d, unsigned mask, const T* in, T* out, int gangs, int workers, int vector,
                        cudaStream_t s) {
@@ -181,6 +233,23 @@ static int paper_typed(const int64_t* d, unsigned mask, const T* in, T* out, int
       count_launch();
       break;
     }
+    case XR_WORKER | XR_VECTOR:
+      paper_wv_kernel<OP, T><<<gangs, block, sb, s>>>(in, out, d[0], d[1], d[2], ifo);
+      count_launch();
+      break;
+    case XR_GANG | XR_WORKER: {
+      void* buf = nullptr;
+      const int64_t rows = (int64_t)gangs * workers, nout = d[2];
+      int st = paper_workspace(s, rows * nout * sizeof(Acc), &buf);
+      if (st) return st;
+      paper_gw_partial_kernel<OP, T><<<gangs, block, 0, s>>>(in, (Acc*)buf, d[0], d[1], d[2]);
+      count_launch();
+      const int nb = 256;
+      paper_second_kernel<OP, T><<<(unsigned)std::min<int64_t>(nout, 65535), nb, nb * sizeof(Acc), s>>>(
+          (const Acc*)buf, rows, nout, out, ifo);
+      count_launch();
+      break;
+    }
     case 7u: {
       void* buf = nullptr;
       const int64_t nth = (int64_t)gangs * workers * vector;
@@ -207,7 +276,7 @@ extern "C" int xr_reduce_paper(int op, int dtype, const int64_t nest_dims[3], un
                                void* out, int num_gangs, int num_workers, int vector_length, xr_stream_t stream) {
   if (!nest_dims || (level_mask & ~(7u | XR_INIT_FROM_OUT)) != 0u) return XR_ERR_INVALID;
   const unsigned m = level_mask & 7u;
-  if (m != XR_GANG && m != XR_WORKER && m != XR_VECTOR && m != 7u) return XR_ERR_UNSUPPORTED;
+  if (m == (XR_GANG | XR_VECTOR) || m == 0u) return XR_ERR_UNSUPPORTED;  // gang & vector: not in the paper
   if (op != XR_OP_ADD && op != XR_OP_MUL && op != XR_OP_MAX) return XR_ERR_UNSUPPORTED;
   if (dtype != XR_INT32 && dtype != XR_FP32 && dtype != XR_FP64) return XR_ERR_UNSUPPORTED;
   for (int d = 0; d < 3; ++d)

@@ -34,7 +34,7 @@ def run_paper(op, dtype, dims, levels, x, init=None, launch=(0, 0, 0)):
 def test_paper_kernels_match_oracle(op, dtype):
     kind = {"+": "ints", "*": "mul", "max": "maxmin"}[op]
     for dims in [(64, 64, 128), (5, 13, 1000), (300, 2, 32), (3, 37, 77)]:
-        for lv in ["g", "w", "v", "gwv"]:
+        for lv in ["g", "w", "v", "gw", "wv", "gwv"]:
             x = recipes.make(kind, dims, oracle.mask_of(lv), dtype, 7)
             init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 8)
             check(op, dtype, dims, lv, run_paper(op, dtype, dims, lv, x, init=init), x, init=init)
@@ -46,10 +46,10 @@ def test_paper_kernels_launch_shapes_and_errors():
     dims = (33, 19, 250)
     x = recipes.make("ints", dims, 7, "int32", 3)
     for launch in [(192, 8, 128), (148 * 16, 4, 256), (7, 1, 32), (1, 32, 32)]:
-        for lv in ["g", "w", "v", "gwv"]:
+        for lv in ["g", "w", "v", "gw", "wv", "gwv"]:
             check("+", "int32", dims, lv, run_paper("+", "int32", dims, lv, x, launch=launch), x)
     t = torch.zeros(8, device="cuda")
     assert xr.xr_reduce_paper("&", "int32", (2, 2, 2), "g", t.data_ptr(), t.data_ptr()) == xr.ERR_UNSUPPORTED
-    assert xr.xr_reduce_paper("+", "fp32", (2, 2, 2), "gw", t.data_ptr(), t.data_ptr()) == xr.ERR_UNSUPPORTED
+    assert xr.xr_reduce_paper("+", "fp32", (2, 2, 2), "gv", t.data_ptr(), t.data_ptr()) == xr.ERR_UNSUPPORTED
     assert xr.xr_reduce_paper("+", "fp32", (2, 2, 2), "g", t.data_ptr(), t.data_ptr(), 4, 3, 100) == \
         xr.ERR_INVALID

@@ -20,10 +20,11 @@ TDT = {"int32": torch.int32, "fp32": torch.float32, "fp64": torch.float64}
 SZ = {"int32": 4, "fp32": 4, "fp64": 8}
 # (label, dims, levels): cfg1; the paper's testsuite sizes (reading C15: the
 # reduced loop 2^20, the other two 2 and 32, outer -> inner); 512^3
-CASES = [("cfg1", (64, 64, 128), lv) for lv in ("g", "w", "v", "gwv")] + [
+CASES = [("cfg1", (64, 64, 128), lv) for lv in ("g", "w", "v", "gw", "wv", "gwv")] + [
     ("paper-1M", (1 << 20, 2, 32), "g"), ("paper-1M", (2, 1 << 20, 32), "w"),
     ("paper-1M", (2, 32, 1 << 20), "v"), ("paper-1M", (1 << 20, 2, 32), "gwv")] + [
-    ("512^3", (512, 512, 512), lv) for lv in ("g", "w", "v", "gwv")]
+    ("paper-1M", (1 << 20, 2, 32), "gw"), ("paper-1M", (2, 1 << 20, 32), "wv")] + [
+    ("512^3", (512, 512, 512), lv) for lv in ("g", "w", "v", "gw", "wv", "gwv")]
 LAUNCHES = {"paper192": (192, 8, 128), "b200": (148 * 8, 8, 128)}
 
 
