@@ -347,6 +347,13 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
 }
 
 // ------------------------------------------------------------- stream kernel
+// The warp-specialised ring kernels (stream, rows, rkr, coltma) run 3 CTAs per
+// SM (64 KiB ring each); declaring that residency lets ptxas keep every
+// shared-memory load of a stage in flight instead of reusing one register
+// quadruple per load (r01 SASS: serialized LDS.128 chains without it).
+#ifndef XR_WS_MINB
+#define XR_WS_MINB 3
+#endif
 // R and long-row KR shapes (C == 1): each unit is one contiguous range; RKR
 // with 16-B aligned rows (C > 1): each unit is a run of whole rows of one
 // output at the row stride, and the stages are filled from the rows'
@@ -394,7 +401,7 @@ __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u)
 }
 
 template <int OP, typename T, int NS, int STAGE>
-__global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant__ SegArgs a) {
+__global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const __grid_constant__ SegArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -407,17 +414,29 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
   __shared__ long long s_units[RING];
   __shared__ Acc smem[32];
   __shared__ int s_last;
+  // per-output gang tier handed to the epilogue warp: a mailbox of RING unit
+  // results (unit id, CTA value), full / free mbarriers per slot
+  __shared__ __align__(8) uint64_t bfull[RING];
+  __shared__ __align__(8) uint64_t bfree[RING];
+  __shared__ long long box_u[RING];
+  __shared__ Acc box_v[RING];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
   const int64_t S = a.Sr * a.Sc;
   const bool whole = (a.O == 1);
+  const bool epi = !whole && S > 1;
 
   if (tid == 0) {
 #pragma unroll
     for (int k = 0; k < NS; ++k) {
       mbar_init(&full[k], 1);
       mbar_init(&empty[k], kConsWarps);
+    }
+#pragma unroll
+    for (int k = 0; k < RING; ++k) {
+      mbar_init(&bfull[k], 1);
+      mbar_init(&bfree[k], 1);
     }
     fence_mbar_init();
   }
@@ -469,6 +488,40 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
     }
     return;
   }
+  if (warp == kConsWarps + 1) {
+    // ---------------- epilogue warp (a4 per output): takes each unit's CTA
+    // value from the mailbox, writes the unit partial, takes the output's
+    // ticket, and the last arriver folds the output's S partials in unit
+    // order.  The fence + atomic round trip no longer stalls the consumers
+    // (r01y: 512^3 32-bit WV lost ~1 us of the whole CTA per unit).
+    if (!epi) return;
+    for (int n = 0;; ++n) {
+      const int slot = n & (RING - 1);
+      mbar_wait(&bfull[slot], (unsigned)((n / RING) & 1));
+      const long long u = box_u[slot];
+      const Acc v = box_v[slot];
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bfree[slot]);
+      if (u < 0) break;
+      const int64_t o = u / S;
+      unsigned t = 0;
+      if (lane == 0) {
+        partials[u] = v;
+        t = ticket_add(&a.tickets[o]);
+      }
+      t = __shfl_sync(0xffffffffu, t, 0);
+      if (t == (unsigned)(S - 1)) {
+        __threadfence();
+        Acc w = fold_partials<OP, T>(partials + o * S, S, lane, 32);
+        w = group_reduce<OP, T, 32>(w);
+        if (lane == 0) {
+          out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+          a.tickets[o] = 0u;
+        }
+      }
+    }
+    return;
+  }
 
   // ---------------- consumer warps
   const int ct = tid - 32, cw = warp - 1;
@@ -496,13 +549,23 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
       if (k > 0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const int64_t bytes = min((int64_t)STAGE, body_bytes - k * STAGE);
       const unsigned char* st = stage_mem + slot * STAGE;
+      if (bytes == STAGE) {  // full stage: all PER shared-memory loads in flight, then fold
+        U128 x[PER];
 #pragma unroll
-      for (int j = 0; j < PER; ++j) {
-        const int off = (ct + j * kConsThreads) * 16;
-        if (off < bytes) {
-          const U128 x = *reinterpret_cast<const U128*>(st + off);
+        for (int j = 0; j < PER; ++j) x[j] = *reinterpret_cast<const U128*>(st + (ct + j * kConsThreads) * 16);
 #pragma unroll
-          for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x, q)));
+        for (int j = 0; j < PER; ++j)
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x[j], q)));
+      } else {
+#pragma unroll
+        for (int j = 0; j < PER; ++j) {
+          const int off = (ct + j * kConsThreads) * 16;
+          if (off < bytes) {
+            const U128 x = *reinterpret_cast<const U128*>(st + off);
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) acc[j][q] = O::combine(acc[j][q], O::lift(unpack<T>(x, q)));
+          }
         }
       }
       fence_proxy_async_smem();  // generic reads before the async refill
@@ -514,31 +577,28 @@ __global__ void __launch_bounds__(kWsBlock) stream_kernel(const __grid_constant_
     for (int j = 0; j < PER; ++j)
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[j][q] = O::identity();
-    v = cons_reduce<OP, T>(v, smem, cw, lane);
+    // smem slots alternate between units: a warp can write unit n+2's slot
+    // only after the barrier of unit n+1, i.e. after warp 0 read unit n's
+    v = cons_reduce<OP, T>(v, smem + (seq & 1) * kConsWarps, cw, lane);
     const int64_t o = geo.o;
     if (whole) {
       if (ct == 0) partials[u] = v;
     } else if (S == 1) {
       if (ct == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
-    } else {
-      if (ct == 0) {
-        partials[u] = v;
-        const unsigned t = ticket_add(&a.tickets[o]);
-        s_last = (t == (unsigned)(S - 1));
-      }
-      cons_sync();
-      if (s_last) {
-        __threadfence();
-        Acc w = fold_partials<OP, T>(partials + o * S, S, ct, kConsThreads);
-        w = cons_reduce<OP, T>(w, smem, cw, lane);
-        if (ct == 0) {
-          out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
-          a.tickets[o] = 0u;
-        }
-      }
+    } else if (ct == 0) {  // hand the unit to the epilogue warp
+      const int slot = seq & (RING - 1);
+      if (seq >= RING) mbar_wait(&bfree[slot], (unsigned)(((seq / RING) - 1) & 1));
+      box_u[slot] = u;
+      box_v[slot] = v;
+      mbar_arrive(&bfull[slot]);
     }
-    cons_sync();
     ++seq;
+  }
+  if (epi && ct == 0) {  // end marker for the epilogue warp
+    const int slot = seq & (RING - 1);
+    if (seq >= RING) mbar_wait(&bfree[slot], (unsigned)(((seq / RING) - 1) & 1));
+    box_u[slot] = -1;
+    mbar_arrive(&bfull[slot]);
   }
   if (whole) {  // a4: one ticket per CTA; the last CTA folds the S unit partials in unit order
     if (ct == 0) {
@@ -870,7 +930,7 @@ __device__ __forceinline__ void rkr_unit(int64_t u, int64_t S, int64_t njb, int6
 }
 
 template <int OP, typename T, int NS>
-__global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ RkrArgs a) {
+__global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __grid_constant__ RkrArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -880,6 +940,12 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
   __shared__ __align__(8) uint64_t full[NS];
   __shared__ __align__(8) uint64_t empty[NS];
   __shared__ long long s_units[RING];
+  // per-output gang tier handed to the epilogue warp: a mailbox of RING units
+  // (unit id + one value per output row of the j-block)
+  __shared__ __align__(8) uint64_t bfull[RING];
+  __shared__ __align__(8) uint64_t bfree[RING];
+  __shared__ long long box_u[RING];
+  __shared__ typename Op<OP, T>::Acc box_v[RING][32];
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   const int64_t row_bytes = a.L * (int64_t)sizeof(T);
@@ -892,6 +958,11 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
     for (int k = 0; k < NS; ++k) {
       mbar_init(&full[k], 1);
       mbar_init(&empty[k], kConsWarps);
+    }
+#pragma unroll
+    for (int k = 0; k < RING; ++k) {
+      mbar_init(&bfull[k], kConsWarps);
+      mbar_init(&bfree[k], 1);
     }
     fence_mbar_init();
   }
@@ -931,11 +1002,52 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
     return;
   }
 
+  Acc* partials = static_cast<Acc*>(a.partials);
+  if (warp == kConsWarps + 1) {
+    // ---------------- epilogue warp (a4 per output, as in stream_kernel): lane
+    // r takes row r's unit value, writes the partial and the output's ticket;
+    // each output whose last unit this was is folded by the whole warp in
+    // split order.  The consumers never wait for a fence + atomic round trip.
+    if (S == 1) return;
+    for (int n = 0;; ++n) {
+      const int slot = n & (RING - 1);
+      mbar_wait(&bfull[slot], (unsigned)((n / RING) & 1));
+      const long long u = box_u[slot];
+      if (u < 0) break;
+      int64_t jb, s;
+      rkr_unit(u, S, a.units / S, &jb, &s);
+      const int nrows = (int)min((int64_t)J, a.K - jb * J);
+      const Acc v = lane < nrows ? box_v[slot][lane] : O::identity();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&bfree[slot]);
+      bool last = false;
+      if (lane < nrows) {
+        const int64_t o = jb * J + lane;
+        partials[o * S + s] = v;
+        last = (ticket_add(&a.tickets[o]) == (unsigned)(S - 1));
+      }
+      unsigned m = __ballot_sync(0xffffffffu, last);
+      if (m) __threadfence();
+      while (m) {
+        const int r = __ffs(m) - 1;
+        m &= m - 1;
+        const int64_t o = jb * J + r;
+        Acc w = fold_partials<OP, T>(partials + o * S, S, lane, 32);
+        w = group_reduce<OP, T, 32>(w);
+        if (lane == 0) {
+          out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
+          a.tickets[o] = 0u;
+        }
+      }
+    }
+    return;
+  }
+
   // ---------------- consumer warps
   const int cw = warp - 1;
   const int rpw = J / kConsWarps;          // rows per warp per stage (1, 2 or 4)
   const int vpl = (int)(row_bytes >> 9);   // 16-B vectors per lane per row (1, 2 or 4)
-  Acc* partials = static_cast<Acc*>(a.partials);
+  const int vsh = __ffs(vpl) - 1;          // rpw * vpl == 4: vector idx -> row idx >> vsh, piece idx & (vpl-1)
   int seq = 0;
   int64_t g = 0;
   while (true) {
@@ -946,26 +1058,34 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
         rkr_unit(u, S, a.units / S, &jb, &s);
     const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
     const int nrows = (int)min((int64_t)J, a.K - jb * J);
-    Acc acc[4][VEC];
+    Acc acc[4][VEC];  // per vector idx (row idx >> vsh, piece idx & (vpl-1))
 #pragma unroll
-    for (int rr = 0; rr < 4; ++rr)
+    for (int idx = 0; idx < 4; ++idx)
 #pragma unroll
-      for (int q = 0; q < VEC; ++q) acc[rr][q] = O::identity();
+      for (int q = 0; q < VEC; ++q) acc[idx][q] = O::identity();
+    const bool full_rows = (nrows == J);
     for (int64_t k = k0; k < k1; ++k, ++g) {
       const int slot = (int)(g % NS);
       if (k > k0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const unsigned char* sm = stage_mem + slot * STAGE;
+      if (full_rows) {  // all 4 shared-memory loads in flight, then fold
+        U128 x[4];
 #pragma unroll
-      for (int rr = 0; rr < 4; ++rr) {
-        const int r = cw * rpw + rr;
-        if (rr < rpw && r < nrows) {
+        for (int idx = 0; idx < 4; ++idx)
+          x[idx] = *reinterpret_cast<const U128*>(sm + ((int64_t)(cw * rpw + (idx >> vsh)) << rshift) +
+                                                  ((idx & (vpl - 1)) * 32 + lane) * 16);
 #pragma unroll
-          for (int kk = 0; kk < 4; ++kk) {
-            if (kk < vpl) {
-              const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + (kk * 32 + lane) * 16);
+        for (int idx = 0; idx < 4; ++idx)
 #pragma unroll
-              for (int q = 0; q < VEC; ++q) acc[rr][q] = O::combine(acc[rr][q], O::lift(unpack<T>(x, q)));
-            }
+          for (int q = 0; q < VEC; ++q) acc[idx][q] = O::combine(acc[idx][q], O::lift(unpack<T>(x[idx], q)));
+      } else {
+#pragma unroll
+        for (int idx = 0; idx < 4; ++idx) {
+          const int r = cw * rpw + (idx >> vsh);
+          if (r < nrows) {
+            const U128 x = *reinterpret_cast<const U128*>(sm + ((int64_t)r << rshift) + ((idx & (vpl - 1)) * 32 + lane) * 16);
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) acc[idx][q] = O::combine(acc[idx][q], O::lift(unpack<T>(x, q)));
           }
         }
       }
@@ -973,37 +1093,39 @@ __global__ void __launch_bounds__(kWsBlock) rkr_kernel(const __grid_constant__ R
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[slot]);  // the stage is consumed into registers
     }
+    const int bslot = seq & (RING - 1);
+    if (S > 1 && seq >= RING && lane == 0) mbar_wait(&bfree[bslot], (unsigned)(((seq / RING) - 1) & 1));
+    __syncwarp();
 #pragma unroll
     for (int rr = 0; rr < 4; ++rr) {
       const int r = cw * rpw + rr;
       if (rr < rpw && r < nrows) {  // warp-uniform
-        Acc v = acc[rr][0];
+        Acc v = O::identity();
 #pragma unroll
-        for (int q = 1; q < VEC; ++q) v = O::combine(v, acc[rr][q]);
+        for (int idx = 0; idx < 4; ++idx)
+          if ((idx >> vsh) == rr)
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) v = O::combine(v, acc[idx][q]);
         v = group_reduce<OP, T, 32>(v);
         const int64_t o = jb * J + r;
         if (S == 1) {
           if (lane == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
-        } else {  // a4: the last unit of output o folds its S partials in split order
-          int last = 0;
-          if (lane == 0) {
-            partials[o * S + s] = v;
-            last = (ticket_add(&a.tickets[o]) == (unsigned)(S - 1));
-          }
-          last = __shfl_sync(0xffffffffu, last, 0);
-          if (last) {
-            __threadfence();
-            Acc w = fold_partials<OP, T>(partials + o * S, S, lane, 32);
-            w = group_reduce<OP, T, 32>(w);
-            if (lane == 0) {
-              out[o] = merge_init<OP, T>(w, out, o, a.init_from_out);
-              a.tickets[o] = 0u;
-            }
-          }
+        } else if (lane == 0) {  // a4 runs in the epilogue warp
+          box_v[bslot][r] = v;
         }
       }
     }
+    if (S > 1 && lane == 0) {
+      if (cw == 0) box_u[bslot] = u;
+      mbar_arrive(&bfull[bslot]);
+    }
     ++seq;
+  }
+  if (S > 1 && lane == 0) {  // end marker for the epilogue warp
+    const int bslot = seq & (RING - 1);
+    if (seq >= RING) mbar_wait(&bfree[bslot], (unsigned)(((seq / RING) - 1) & 1));
+    if (cw == 0) box_u[bslot] = -1;
+    mbar_arrive(&bfull[bslot]);
   }
 }
 
@@ -1148,7 +1270,7 @@ __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_co
 // tier is the per-tile ticket of col_kernel.  OOB rows/columns of a box are
 // skipped by the consumers, so the fill value never matters.
 template <int OP, typename T, int NS>
-__global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
+__global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int BLOCK = kConsThreads;        // consumer threads
@@ -1243,13 +1365,23 @@ __global__ void __launch_bounds__(kWsBlock) coltma_kernel(const __grid_constant_
       if (k > 0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
       const unsigned char* st = stage_mem + slot * kStageBytes;
       const int64_t rbase = r0 + k * BR;
+      if (col_ok && rbase + BR <= r1) {  // full box: all BR / NPH loads in flight, then fold
+        U128 x[BR / NPH];
 #pragma unroll
-      for (int i = 0; i < BR / NPH; ++i) {
-        const int row = ph + i * NPH;
-        if (col_ok && rbase + row < r1) {
-          const U128 x = *reinterpret_cast<const U128*>(st + row * 1024 + grp * 16);
+        for (int i = 0; i < BR / NPH; ++i) x[i] = *reinterpret_cast<const U128*>(st + (ph + i * NPH) * 1024 + grp * 16);
 #pragma unroll
-          for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
+        for (int i = 0; i < BR / NPH; ++i)
+#pragma unroll
+          for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x[i], q)));
+      } else {
+#pragma unroll
+        for (int i = 0; i < BR / NPH; ++i) {
+          const int row = ph + i * NPH;
+          if (col_ok && rbase + row < r1) {
+            const U128 x = *reinterpret_cast<const U128*>(st + row * 1024 + grp * 16);
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
+          }
         }
       }
       fence_proxy_async_smem();  // generic reads before the async refill
@@ -1419,10 +1551,10 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       static int occ = [&] {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsEpiBlock, dyn) != cudaSuccess || n < 1) n = 1;
         return n;
       }();
-      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsBlock, dyn, s>>>(p.seg);
+      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsEpiBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_RKR: {
@@ -1431,12 +1563,12 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       static int occ = [&] {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
         int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsEpiBlock, dyn) != cudaSuccess || n < 1) n = 1;
         return n;
       }();
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.rkr);
+      kern<<<(unsigned)grid, kWsEpiBlock, dyn, s>>>(p.rkr);
       break;
     }
     case K_ROWS: {

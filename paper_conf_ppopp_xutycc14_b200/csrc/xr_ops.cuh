@@ -105,6 +105,7 @@ namespace xr {
 constexpr int kConsWarps = 8;
 constexpr int kConsThreads = 32 * kConsWarps;
 constexpr int kWsBlock = kConsThreads + 32;  // + the producer warp
+constexpr int kWsEpiBlock = kWsBlock + 32;   // + an epilogue warp (stream kernel)
 
 // Order this thread's generic-proxy shared-memory accesses before later
 // async-proxy (bulk copy / TMA) accesses to the same memory: a consumer
