@@ -13,10 +13,12 @@ import subprocess
 import sys
 
 LDG128 = re.compile(r"\bLDG\.E[.A-Z0-9_:]*\.128")
+LDS128 = re.compile(r"\bLDS(\.U)?\.128")  # shared-memory stage folds of the ring kernels
 
 
-def batches(so: str) -> dict:
-    """{demangled kernel name: (max batch, number of LDG.128)} for kernels with 16-B loads."""
+def batches(so: str, load=LDG128) -> dict:
+    """{demangled kernel name: (max batch, number of 16-B loads)} for kernels with 16-B loads
+    (global LDG.128 by default, LDS128 for shared memory)."""
     txt = subprocess.run(["cuobjdump", "-sass", so], capture_output=True, text=True, check=True).stdout
     func = None
     insts = {}
@@ -32,17 +34,17 @@ def batches(so: str) -> dict:
     names = subprocess.run(["c++filt"], input="\n".join(insts), capture_output=True, text=True).stdout.splitlines()
     out = {}
     for (f, ins), name in zip(insts.items(), names):
-        idx = [i for i, s in enumerate(ins) if LDG128.search(s)]
+        idx = [i for i, s in enumerate(ins) if load.search(s)]
         if not idx:
             continue
         best = 0
         for i in idx:
-            dst = re.search(r"LDG\S*\s+(R\d+)", ins[i]).group(1)
+            dst = re.search(r"LD[GS]\S*\s+(R\d+)", ins[i]).group(1)
             n = 1
             for s in ins[i + 1:i + 40]:
                 parts = s.split(None, 1)
                 ops = parts[1] if len(parts) > 1 else ""
-                if LDG128.search(s):
+                if load.search(s):
                     if re.search(r"\s" + dst + r"\b", s.split(",", 1)[0]):
                         break  # the destination is overwritten by the next load
                     n += 1
