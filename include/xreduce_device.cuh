@@ -62,7 +62,7 @@ template <> __device__ __forceinline__ double highest<double>() { return __longl
 //   int  + * & | ^ : unsigned of the same width (two's-complement wrap, C6)
 //   int  max min   : the signed type
 //   fp   + * max min : the type itself (C23: accumulate in dtype)
-//   && ||          : uint32 truth value (C8)
+//   && ||          : uint32, nonzero = true (C8; see Logical)
 template <int OP, typename T, bool FP = IsFp<T>::value> struct Op;
 
 // ---- integers: + * & | ^
@@ -151,12 +151,28 @@ template <typename T> struct Op<OP_MIN, T, true> {
 };
 
 // ---- && ||  on any type (truth = x != 0: fp NaN true, +-0 false; C8)
+// The accumulator is a uint32 whose truth is "nonzero" (not 0/1): lift keeps
+// the magnitude bits (fp: sign cleared, so +-0 -> 0 and NaN -> nonzero; 64-bit:
+// low | high word), && combines by unsigned min (zero wins), || by OR.  One
+// LOP3 / IMNMX per element in the fold instead of a compare + select + logic op.
+template <typename T> __device__ __forceinline__ uint32_t truth_bits(T x) {
+  if constexpr (sizeof(T) == 4) {
+    uint32_t u;
+    memcpy(&u, &x, 4);
+    return IsFp<T>::value ? (u & 0x7fffffffu) : u;
+  } else {
+    unsigned long long u;
+    memcpy(&u, &x, 8);
+    const uint32_t lo = (uint32_t)u, hi = (uint32_t)(u >> 32);
+    return lo | (IsFp<T>::value ? (hi & 0x7fffffffu) : hi);
+  }
+}
 template <int OP, typename T> struct Logical {
   using Acc = uint32_t;
-  static __device__ __forceinline__ Acc identity() { return OP == OP_LAND ? 1u : 0u; }
-  static __device__ __forceinline__ Acc lift(T x) { return x != T(0) ? 1u : 0u; }
+  static __device__ __forceinline__ Acc identity() { return OP == OP_LAND ? 0xffffffffu : 0u; }
+  static __device__ __forceinline__ Acc lift(T x) { return truth_bits<T>(x); }
   static __device__ __forceinline__ Acc combine(Acc a, Acc b) {
-    return OP == OP_LAND ? (a & b) : (a | b);
+    return OP == OP_LAND ? (a < b ? a : b) : (a | b);
   }
   static __device__ __forceinline__ T finish(Acc a) { return a ? T(1) : T(0); }
 };

@@ -120,6 +120,47 @@ def test_fp_special_values(op, dtype, staging):
         check(op, dtype, (3, 1, 1), "g", gpu_reduce(op, dtype, (3, 1, 1), "g", z), z)
 
 
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("op", ["&&", "||"])
+def test_logical_truth_bit_patterns(op, dtype, staging):
+    """C8 truth (x != 0) on the bit patterns the kernels' nonzero-accumulator
+    folds must classify: sign-only words (INT_MIN, -0.0), 64-bit values whose
+    low or high word alone is nonzero (2^32, 1, subnormals), NaN payloads.
+    Inputs: all truthy (&& -> 1), all falsy (|| -> 0), and sparse mixes."""
+    rng = np.random.default_rng(808)
+    npdt = oracle.NP_DTYPES[dtype]
+    if dtype == "int32":
+        truthy = np.array([np.iinfo(np.int32).min, 1, -1, 1 << 16, (1 << 31) - 1], dtype=np.int64).astype(np.int32)
+        falsy = np.zeros(1, np.int32)
+    elif dtype == "int64":
+        truthy = np.array([np.iinfo(np.int64).min, 1 << 32, -(1 << 32), 1, (1 << 63) - 1, 0x80000000], dtype=np.int64)
+        falsy = np.zeros(1, np.int64)
+    else:
+        ut = np.uint32 if dtype == "fp32" else np.uint64
+        sign = ut(1) << ut(31 if dtype == "fp32" else 63)
+        pats = [1, sign | ut(1), (ut(0xFF) << ut(23)) | ut(1) if dtype == "fp32" else (ut(0x7FF) << ut(52)) | ut(1)]
+        if dtype == "fp64":
+            pats += [ut(1) << ut(32), sign | (ut(1) << ut(32))]  # high word only (low word zero)
+        truthy = np.array(pats, dtype=ut).view(npdt)
+        falsy = np.array([0, sign], dtype=ut).view(npdt)  # +0, -0
+    for dims in [(5, 7, 300), (3, 130, 33)]:
+        n = int(np.prod(dims))
+        for kind in ("truthy", "falsy", "mix"):
+            if kind == "truthy":
+                x = rng.choice(truthy, n)
+            elif kind == "falsy":
+                x = rng.choice(falsy, n)
+            else:
+                x = rng.choice(truthy, n)
+                x[rng.random(n) < 0.002] = falsy[-1]
+                y = rng.choice(falsy, n)
+                y[rng.random(n) < 0.002] = truthy[0]
+                x = y if op == "||" else x  # sparse truthy in falsy for ||, the reverse for &&
+            x = np.ascontiguousarray(x.astype(npdt, copy=False))
+            for levels in ALL_MASKS:
+                check(op, dtype, dims, levels, gpu_reduce(op, dtype, dims, levels, x), x)
+
+
 # ---------------------------------------------------------------- fuzz: ragged, misaligned
 def test_fuzz_shapes_and_misalignment(staging):
     rng = random.Random(2014)
