@@ -45,3 +45,41 @@ def test_ring_stage_folds_keep_four_smem_loads_in_flight():
     bad = {n: b for n, b in checked.items() if b < 2}
     assert not bad, bad
     assert sum(b >= 4 for b in checked.values()) >= 0.75 * len(checked), sorted(checked.values())
+
+
+def _sass_by_kernel(so):
+    import re
+    import subprocess
+    txt = subprocess.run(["cuobjdump", "-sass", so], capture_output=True, text=True, check=True).stdout
+    func, insts = None, {}
+    for line in txt.splitlines():
+        m = re.match(r"\s+Function : (\S+)", line)
+        if m:
+            func = m.group(1)
+            insts[func] = []
+            continue
+        m = re.match(r"\s+/\*[0-9a-f]+\*/\s+(.*?);", line)
+        if m and func:
+            insts[func].append(m.group(1))
+    names = subprocess.run(["c++filt"], input="\n".join(insts), capture_output=True, text=True).stdout.splitlines()
+    return dict(zip(names, insts.values()))
+
+
+@pytest.mark.skipif(shutil.which("cuobjdump") is None, reason="cuobjdump not on PATH")
+def test_logical_and_folds_use_unsigned_min():
+    """`&&` accumulates a nonzero-truth u32 folded by unsigned min (DESIGN.md
+    section 5): the 32-bit ring kernels must fold with IMNMX(3).U32 and stay
+    within 15 % of the static size of the `+` instantiation (the old 0/1 lift
+    cost a compare + select + logic op per element)."""
+    k = _sass_by_kernel(SO)
+    checked = 0
+    for fam in ("xr::stream_kernel<", "xr::rkr_kernel<", "xr::coltma_kernel<"):
+        for dt in ("int", "float"):
+            land = [n for n in k if n.startswith("void " + fam + "7, " + dt + ",")]
+            for n in land:
+                add = n.replace(fam + "7, ", fam + "0, ", 1)
+                assert any("IMNMX" in s and ".U32" in s for s in k[n]), n
+                if add in k:
+                    assert len(k[n]) <= 1.15 * len(k[add]), (n, len(k[n]), len(k[add]))
+                checked += 1
+    assert checked >= 6, checked
