@@ -162,6 +162,7 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
 // columns are ~3% extra).
 constexpr int kTileCols = 2 * kConsThreads;    // 512 doubles = 4 KiB per row
 constexpr int kSlotDoubles = kTileCols + 4;    // + 2-column halo on both sides
+constexpr int kSlotDoublesP = kTileCols + 8;   // persistent kernel: + 2 lead + 1 shift, 16-B rows
 constexpr int kHeatSlots = 8;
 
 __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
@@ -276,10 +277,14 @@ struct HeatPArgs {
   unsigned long long* sched;    // [2] tile counter + exit counter
 };
 
-__global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa) {
+template <bool ODD>  // ODD: ni odd, rows staged with a per-row 8-B shift
+__global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(HeatPArgs pa) {
   using O = Op<OP_MAX, double>;
   constexpr int RING = 8;
-  __shared__ __align__(128) double slots[kHeatSlots][kSlotDoubles];
+  // Row layout: global column c of a row staged from element e0 = ws - sh
+  // (sh = 1 when the window start is not 16-B aligned, odd ni) sits at index
+  // c - c0 + 4 + sh; rows stay 16-B aligned for the bulk copies.
+  __shared__ __align__(128) double slots[kHeatSlots][kSlotDoublesP];
   __shared__ __align__(8) uint64_t full[kHeatSlots];
   __shared__ __align__(8) uint64_t empty[kHeatSlots];
   __shared__ long long s_tiles[RING];
@@ -320,13 +325,23 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
         int64_t c0, j0, j1;
         tile_geom(t, &c0, &j0, &j1);
         const int64_t ws = max(c0 - 2, (int64_t)0), we = min(c0 + kTileCols + 2, ni);
-        const unsigned wbytes = (unsigned)((we - ws) * 8);
         const int64_t soff = ws - (c0 - 2);
+        const int64_t total = a.nj * ni;
         for (int64_t r = 0; r < j1 - j0 + 2; ++r, ++q) {  // rows j0-1 .. j1
           const int slot = (int)(q % kHeatSlots);
+          const int64_t e = (j0 - 1 + r) * ni + ws;
+          int64_t sh = 0, cnt = we - ws;
+          if constexpr (ODD) {
+            sh = e & 1;                                  // T1 is 16-B aligned
+            cnt = (we - ws + sh + 1) & ~(int64_t)1;      // whole 16-B pairs
+            // never past the buffer: the dropped element is then the last column
+            // of the buffer's last row, which only serves as a (boundary) halo value
+            if (e - sh + cnt > total) cnt -= 2;
+          }
+          const unsigned wbytes = (unsigned)(cnt * 8);
           if (q >= kHeatSlots) mbar_wait(&empty[slot], (unsigned)(((q / kHeatSlots) - 1) & 1));
           mbar_expect_tx(&full[slot], wbytes);
-          bulk_g2s(&slots[slot][soff], a.T1 + (j0 - 1 + r) * ni + ws, wbytes, &full[slot]);
+          bulk_g2s(&slots[slot][soff + 2], a.T1 + e - sh, wbytes, &full[slot]);
         }
         t = nt;
       }
@@ -350,9 +365,11 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
     const int64_t qb = q;  // global index of row 0 of this tile
     mbar_wait(&full[(qb + 1) % kHeatSlots], (unsigned)(((qb + 1) / kHeatSlots) & 1));
     const int64_t col = c0 + 2 * tid;
-    const int li = 2 + 2 * tid;
+    const int li = 4 + 2 * tid;
     const bool i0 = col >= 1 && col <= ni - 2;
     const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
+    const int64_t ws = max(c0 - 2, (int64_t)0);
+    constexpr bool odd = ODD;
     for (int64_t r = 1; r < nrows - 1; ++r) {
       const int64_t qd = qb + r + 1;
       mbar_wait(&full[qd % kHeatSlots], (unsigned)((qd / kHeatSlots) & 1));
@@ -360,19 +377,31 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
         const double* up = slots[(qb + r - 1) % kHeatSlots];
         const double* cur = slots[(qb + r) % kHeatSlots];
         const double* dn = slots[qd % kHeatSlots];
-        const double2 u2 = *reinterpret_cast<const double2*>(up + li);
-        const double2 c2 = *reinterpret_cast<const double2*>(cur + li);
-        const double2 d2 = *reinterpret_cast<const double2*>(dn + li);
-        const double l = cur[li - 1], rr = cur[li + 2];
+        const int64_t ecur = (j0 - 1 + r) * ni + ws;  // window start element of row r
+        double2 u2, c2, d2;
+        double l, rr;
+        if constexpr (!odd) {  // every row 16-B aligned: vector loads
+          u2 = *reinterpret_cast<const double2*>(up + li);
+          c2 = *reinterpret_cast<const double2*>(cur + li);
+          d2 = *reinterpret_cast<const double2*>(dn + li);
+          l = cur[li - 1];
+          rr = cur[li + 2];
+        } else {  // rows alternate the staging shift (ni odd)
+          const int su = li + (int)((ecur - ni) & 1), sc = li + (int)(ecur & 1), sd = li + (int)((ecur + ni) & 1);
+          u2 = make_double2(up[su], up[su + 1]);
+          c2 = make_double2(cur[sc], cur[sc + 1]);
+          d2 = make_double2(dn[sd], dn[sd + 1]);
+          l = cur[sc - 1];
+          rr = cur[sc + 2];
+        }
         const double n0 = stencil(u2.x, d2.x, l, c2.y);
         const double n1 = stencil(u2.y, d2.y, c2.x, rr);
         double* dst = a.T2 + (j0 + r - 1) * ni + col;
-        if (i0 && i1) {
+        if (i0 && i1 && !(odd && (((uintptr_t)dst) & 15u))) {
           __stcs(reinterpret_cast<double2*>(dst), make_double2(n0, n1));
-        } else if (i0) {
-          __stcs(dst, n0);
         } else {
-          __stcs(dst + 1, n1);
+          if (i0) __stcs(dst, n0);
+          if (i1) __stcs(dst + 1, n1);
         }
         if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
         if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
@@ -410,8 +439,12 @@ __global__ void __launch_bounds__(kWsBlock) heat_persistent_kernel(HeatPArgs pa)
 // Sweep output rows [jb, je) of an nj x ni buffer (rows jb-1 and je are read).
 static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
                        double* residual, cudaStream_t s) {
-  const bool v2 = (ni % 2 == 0) && ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
-  const bool bulk = v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr;
+  const bool al16 = ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
+  const bool v2 = (ni % 2 == 0) && al16;
+  // odd ni: only the persistent kernel stages rows with a per-row 8-B shift
+  const bool odd_bulk = (ni % 2 == 1) && al16 && ni >= 5 && je > jb && std::getenv("XR_NO_BULK") == nullptr &&
+                        std::getenv("XR_HEAT_ONE_TILE") == nullptr && std::getenv("XR_NO_ODD_BULK") == nullptr;
+  const bool bulk = (v2 && ni >= 4 && std::getenv("XR_NO_BULK") == nullptr) || odd_bulk;
   const int strip = bulk ? kTileCols : 32 * (v2 ? 2 : 1) * (kBlock / 32);
   const int64_t gx = (ni + strip - 1) / strip;
   // 64-row tiles (one tile per CTA: 2048 CTAs at 8192^2; the persistent kernel
@@ -438,12 +471,15 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   dim3 grid((unsigned)gx, (unsigned)gy);
   const char* hp = std::getenv("XR_HEAT_ONE_TILE");  // A/B: one tile per CTA
   if (bulk && hp == nullptr && je > jb) {
-    static int occ = [] {
+    auto occ_of = [](auto kern) {
       int n = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, heat_persistent_kernel, kWsBlock, 0) != cudaSuccess || n < 1)
-        n = 1;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, 0) != cudaSuccess || n < 1) n = 1;
       return n;
-    }();
+    };
+    static const int occ_even = occ_of(heat_persistent_kernel<false>);
+    static const int occ_odd = occ_of(heat_persistent_kernel<true>);
+    const bool odd = (ni % 2) != 0;
+    const int occ = odd ? occ_odd : occ_even;
     int dev = 0, sms = 148;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     HeatPArgs pa;
@@ -452,7 +488,8 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
     pa.gy = gy;
     pa.sched = reinterpret_cast<unsigned long long*>(tickets + 2);  // after the residual ticket (8-B aligned)
     const int64_t pgrid = std::min<int64_t>(gx * gy, (int64_t)sms * occ);
-    heat_persistent_kernel<<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
+    if (odd) heat_persistent_kernel<true><<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
+    else heat_persistent_kernel<false><<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
   } else if (bulk) heat_bulk_kernel<<<grid, kWsBlock, 0, s>>>(a);
   else if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
   else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);

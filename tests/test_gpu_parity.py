@@ -269,7 +269,7 @@ def test_launch_count_single_pass():
 
 
 # ---------------------------------------------------------------- heat (config 4)
-@pytest.mark.parametrize("nj,ni", [(8, 8), (130, 258), (67, 131), (3, 40), (300, 64)])
+@pytest.mark.parametrize("nj,ni", [(8, 8), (130, 258), (67, 131), (3, 40), (300, 64), (9, 5), (41, 1027), (20, 515), (7, 2049)])
 def test_heat_bitwise(nj, ni):
     import torch
     import paper_conf_ppopp_xutycc14_b200 as xr

@@ -148,7 +148,7 @@ def run_xform(name, reps, timed):
                           "elements_per_s": n / med * 1e3}), flush=True)
 
 
-def run_heat(reps, timed, n=8192):
+def run_heat(reps, timed, n=8192, case="cfg4-heat"):
     t1 = torch.zeros(n * n, dtype=torch.float64, device="cuda")
     t1[:n] = 1.0
     t2 = t1.clone()
@@ -168,7 +168,7 @@ def run_heat(reps, timed, n=8192):
         ms = sorted(a.elapsed_time(b) for a, b in evs)
         med = ms[len(ms) // 2]
         byts = 16 * n * n
-        print(json.dumps({"case": "cfg4-heat", "dims": [n, n], "ms_median": med, "ms_min": ms[0],
+        print(json.dumps({"case": case, "dims": [n, n], "ms_median": med, "ms_min": ms[0],
                           "bytes": byts, "GBps": byts / med / 1e6, "frac_of_peak": byts / med / 1e6 / peak(),
                           "points_per_s": n * n / med * 1e3}), flush=True)
 
@@ -184,6 +184,9 @@ def main():
     for name in a.case:
         if name == "cfg4-heat":
             run_heat(a.reps, a.time)
+            continue
+        if name.startswith("heat-"):  # heat-<n>: an n x n grid (odd n: the shifted-staging path)
+            run_heat(a.reps, a.time, int(name.split("-")[1]), name)
             continue
         if name.startswith("mc-pi") or name == "dot-rows":
             run_xform(name, a.reps, a.time)
