@@ -32,7 +32,7 @@ for op, dtype, dims, lv in cases:
                       "|": "bor"}[op], dims, oracle.mask_of(lv), dtype, 1)
     check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
 # heat (bulk + register variants), transform-reduce, multi, paper kernels
-for nj, ni in [(70, 1030), (33, 67)]:
+for nj, ni in [(70, 1030), (33, 67), (9, 5), (41, 1027)]:  # odd ni: shifted bulk staging (clip at the buffer end)
     T0 = oracle.heat_init(nj, ni)
     t1 = torch.from_numpy(T0).cuda()
     t2 = t1.clone()
