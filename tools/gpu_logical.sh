@@ -2,8 +2,8 @@
 # && || accumulator as "nonzero" truth (umin / OR folds): parity (full GPU suite) + the logical cfg5 cells
 mkdir -p gpurun_out
 TAG=${TAG:-logical}
-CASES=""
-for op in '&&' '||' '+' '|'; do for dt in int32 fp32 int64 fp64; do for lv in g w v gw gv wv gwv; do CASES="$CASES cfg5-$op-$dt-$lv"; done; done; done
+
+CASES=cfg5-all
 timeout 900 python tools/kdriver.py $CASES --reps 15 --time > gpurun_out/cfg5_$TAG.jsonl 2>&1
 timeout 2400 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu_$TAG.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu_$TAG.log
 timeout 600 python bench.py > gpurun_out/bench_$TAG.json 2> gpurun_out/bench_$TAG.err
