@@ -11,6 +11,9 @@ BASELINE cfg2 reading "1 GPU then sharded 2/4/8 GPUs"), and one step =
 xr_reduce_sharded (local single-pass kernel + one cross-GPU combine: the fused
 NVLink mailbox exchange inside the same kernel, or one NCCL allreduce).
 --scaling weak gives every rank its own 2^30-element slice instead.
+`--gpus N` without torchrun (WORLD_SIZE unset) re-launches this script under
+torch.distributed.run with N ranks; fewer than N visible GPUs is an error
+(exit 2), and so is a WORLD_SIZE that differs from --gpus.
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference]
                   [--scaling strong|weak]
@@ -66,6 +69,46 @@ def parse():
     ap.add_argument("--force-comm", action="store_true",
                     help="use the NCCL sharded path even at world size 1 (exercises xr_comm_*)")
     return ap.parse_args()
+
+
+def free_port() -> int:
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
+def launch_ranks(args):
+    """--gpus N > 1 outside torchrun: spawn the N ranks ourselves (one process
+    per GPU, NCCL over NVLink).  Returns the exit code, or None to run here."""
+    world_env = os.environ.get("WORLD_SIZE")
+    if world_env is not None:
+        if int(world_env) != args.gpus:
+            sys.stderr.write(f"bench.py: WORLD_SIZE={world_env} but --gpus {args.gpus}; launch one rank per GPU "
+                             f"(torchrun --nproc-per-node {args.gpus}) or drop --gpus\n")
+            return 2
+        return None
+    if args.gpus <= 1 or args.impl == "reference":
+        return None
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        sys.stderr.write(f"bench.py: --gpus {args.gpus} needs {args.gpus} visible GPUs, this host has {have}\n")
+        return 2
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
+def cpu_model() -> str:
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def dist_env():
@@ -153,13 +196,14 @@ def peak_hbm():
         return FALLBACK_HBM_GBS, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def ncu_traffic(wl):
-    """dram bytes per launch of the dominant kernel from the committed ncu capture."""
-    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+def ncu_record(wl):
+    """The committed ncu capture of this workload's kernel (profiles/ncu_dram.json,
+    written by tools/ncu_summary.py): DRAM bytes per launch and
+    dram__throughput.avg.pct_of_peak_sustained_elapsed, with its source."""
+    p = os.path.join(ROOT, "profiles", "ncu_dram.json")
     try:
         with open(p) as f:
-            d = json.load(f)
-        return d.get(wl)
+            return json.load(f).get(wl)
     except Exception:
         return None
 
@@ -226,6 +270,51 @@ def run_reference(args):
 
 
 # --------------------------------------------------------------------- GPU arm
+def timed_loop(step, steps, stream, world):
+    """K steps bracketed by barrier + synchronize; returns (max-over-ranks ms
+    of the whole loop, per-step event ms on this rank)."""
+    import torch
+    import torch.distributed as dist
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0.record(stream)
+    for i in range(steps):
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    total = t0.elapsed_time(t1)
+    if world > 1:
+        t = torch.tensor([total], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        total = float(t.item())
+    return total, [x.elapsed_time(y) for x, y in ev]
+
+
+def pinned_h2d_gbs(host, dev, reps=3):
+    """Measured pinned host -> device copy bandwidth (the e2e ceiling)."""
+    import torch
+    s = torch.cuda.current_stream()
+    best = None
+    for _ in range(reps):
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(s)
+        dev.copy_(host, non_blocking=True)
+        b.record(s)
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b)
+        best = ms if best is None else min(best, ms)
+    return host.numel() * host.element_size() / (best / 1e3) / 1e9
+
+
 def run_gpu(args):
     import torch
     import torch.distributed as dist
@@ -259,13 +348,19 @@ def run_gpu(args):
     stream = torch.cuda.current_stream()
     sh = stream.cuda_stream
     comm = xr.Comm() if use_comm else None
+    if use_comm:
+        dist.barrier()  # ranks arrive together at the first (fused) exchange
+
+    def local_step():
+        st = xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), sh)
+        if st != 0:
+            raise xr.XReduceError(st, "bench local step")
 
     def step():
         if comm is None:
-            st = xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), sh)
-        else:
-            st = xr._lib.xr_reduce_sharded(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)), xr.mask_of("gwv"),
-                                           x.data_ptr(), out.data_ptr(), comm.handle, sh)
+            return local_step()
+        st = xr._lib.xr_reduce_sharded(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)), xr.mask_of("gwv"),
+                                       x.data_ptr(), out.data_ptr(), comm.handle, sh)
         if st != 0:
             raise xr.XReduceError(st, "bench step")
 
@@ -277,7 +372,8 @@ def run_gpu(args):
         # the fused exchange (local reduction + NVLink peer mailboxes in ONE
         # kernel) must agree with the NCCL path; otherwise fall back to NCCL
         q = comm.query()
-        exchange = "fused-nvlink-mailbox" if q["fused"] else "nccl"
+        exchange = "fused NVLink peer-mailbox exchange inside the reduction kernel" if q["fused"] else \
+            "ncclAllReduce after the local kernel"
         if q["fused"]:
             step()
             torch.cuda.synchronize()
@@ -291,9 +387,9 @@ def run_gpu(args):
             flag = torch.tensor([1 if (ok and comm.query()["status"] == 0) else 0], device="cuda")
             dist.all_reduce(flag, op=dist.ReduceOp.MIN)
             if int(flag.item()) == 1:
-                comm.set_fused(True)
+                comm.set_fused(True)  # collective: every rank takes this branch
             else:
-                exchange = "nccl (fused exchange disagreed or timed out; disabled)"
+                exchange = "ncclAllReduce after the local kernel (fused exchange disagreed or timed out; disabled)"
             for _ in range(3):
                 step()
             torch.cuda.synchronize()
@@ -301,105 +397,126 @@ def run_gpu(args):
     clocks = ClockSampler(local)
     clocks.start()
     time.sleep(0.3)  # let the sampler attach
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    if use_comm:
-        dist.barrier()
-    torch.cuda.synchronize()
     launches0 = xr.xr_launch_count()
-    t_start = torch.cuda.Event(enable_timing=True)
-    t_end = torch.cuda.Event(enable_timing=True)
-    t_start.record(stream)
-    for i in range(args.steps):
-        ev[i][0].record(stream)
-        step()
-        ev[i][1].record(stream)
-    t_end.record(stream)
-    torch.cuda.synchronize()
-    if use_comm:
-        dist.barrier()
+    total_ms, per = timed_loop(step, args.steps, stream, world)
     launches = xr.xr_launch_count() - launches0
     ck = clocks.stop()
-    total_ms = t_start.elapsed_time(t_end)
-    per = [a.elapsed_time(b) for a, b in ev]
-    if use_comm:
-        t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
     ms_step = total_ms / args.steps
     value = total * args.steps / (total_ms / 1e3)
 
-    # kernel-only duration: at N=1 the step IS the one reduction kernel
+    # kernel-only duration on this rank: at N=1 the step IS the one reduction
+    # kernel; at N>1 the local kernel is timed alone as well (no exchange)
     kern_ms = statistics.mean(per)
-    plan = xr.xr_plan_describe(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), torch.cuda.get_device_properties(0).multi_processor_count)
+    multi = None
+    if use_comm:  # N>1 (or --force-comm at N=1, which exercises the same code)
+        loc_total, loc_per = timed_loop(local_step, args.steps, stream, world)
+        kern_ms = statistics.mean(loc_per)
+        # 1-GPU reference time in the same run: rank 0 reduces the whole
+        # strong-scaling array (its own slice repeated: timing does not depend
+        # on the values) or, weak, its own slice
+        t1_ms = None
+        if rank == 0:
+            if args.scaling == "strong":
+                xf = x.repeat(world)
+                of = torch.zeros(1, dtype=tdt, device="cuda")
+
+                def full_step():
+                    st = xr.xr_reduce(op, dtype, (total, 1, 1), "gwv", xf.data_ptr(), of.data_ptr(), sh)
+                    if st != 0:
+                        raise xr.XReduceError(st, "bench 1-GPU reference step")
+                for _ in range(3):
+                    full_step()
+                t1_total, _ = timed_loop(full_step, args.steps, stream, 1)
+                t1_ms = t1_total / args.steps
+                del xf
+            else:
+                t1_ms = loc_total / args.steps
+        peak0, _ = peak_hbm()
+        multi = {
+            "exchange": exchange,
+            "kernel_only_ms_per_step": loc_total / args.steps,
+            "kernel_plus_exchange_ms_per_step": ms_step,
+            "exchange_ms_per_step": ms_step - loc_total / args.steps,
+            "aggregate_elements_per_s": value,
+            "aggregate_roofline": {"achieved_gbs": total * esz / (ms_step / 1e3) / 1e9,
+                                   "peak_gbs": world * peak0,
+                                   "frac": total * esz / (ms_step / 1e3) / 1e9 / (world * peak0)},
+            "one_gpu_ms_same_run": t1_ms,
+            "efficiency_t1_over_n_tn": (t1_ms / (world * ms_step)) if (t1_ms and args.scaling == "strong")
+            else (t1_ms / ms_step if t1_ms else None),
+            "timing": "CUDA events on each rank, barrier + synchronize around the loop, max over ranks",
+        }
+    plan = xr.xr_plan_describe(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), torch.cuda.get_device_properties(local).multi_processor_count)
     kernel_name = {"stream": "stream_kernel (cp.async.bulk smem ring, single pass)",
                    "seg": "seg_kernel", "col": "col_kernel", "coltma": "coltma_kernel"}.get(plan["kernel"], plan["kernel"]) + \
         f" [{plan['shape']} shape, {plan['units']} units, grid {plan['grid']}]"
     peak, peak_src = peak_hbm()
     alg_bytes = n * esz + esz  # read every input element once + write one output
     achieved = alg_bytes / (kern_ms / 1e3) / 1e9
-    traffic = ncu_traffic(wl)
+    ncu = ncu_record(wl)
 
     # e2e through the C ABI with HOST buffers (H2D of the step's input + D2H of the result)
     e2e = None
     if args.e2e_steps > 0:
         out_h = np.zeros(1, dtype={"fp32": np.float32, "int64": np.int64}[dtype])
         hp = host.data_ptr()
-        if comm is None:
-            xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)  # warm staging
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            for _ in range(args.e2e_steps):
-                st = xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)
-                assert st == 0
-            el = time.perf_counter() - t0
-        else:
-            dev = torch.empty_like(x)
-            outd = torch.zeros(1, dtype=tdt, device="cuda")
+
+        def host_call():
+            if comm is None:
+                return xr.xr_reduce_host(op, dtype, (n, 1, 1), "gwv", hp, out_h.ctypes.data, sh)
+            return xr._lib.xr_reduce_sharded_host(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)),
+                                                  xr.mask_of("gwv"), hp, out_h.ctypes.data, comm.handle, sh)
+        assert host_call() == 0  # warm the staging buffers
+        if world > 1:
             dist.barrier()
-            t0 = time.perf_counter()
-            for _ in range(args.e2e_steps):
-                dev.copy_(host, non_blocking=True)
-                st = xr._lib.xr_reduce_sharded(xr.OPS[op], xr.DTYPES[dtype], xr._dims((n, 1, 1)), xr.mask_of("gwv"),
-                                               dev.data_ptr(), outd.data_ptr(), comm.handle, sh)
-                assert st == 0
-                outd.cpu()
-            torch.cuda.synchronize()
-            el = time.perf_counter() - t0
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            st = host_call()
+            assert st == 0, st
+        el = time.perf_counter() - t0
+        if world > 1:
             t = torch.tensor([el], dtype=torch.float64, device="cuda")
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             el = float(t.item())
+        h2d = pinned_h2d_gbs(host, x)
         e2e = {"value": total * args.e2e_steps / el, "unit": "elements/s",
                "h2d_bytes_per_step": n * esz, "d2h_bytes_per_step": esz, "steps": args.e2e_steps,
-               "api": "xr_reduce_host (C ABI, pinned host input)" if world == 1 else
-                      "pinned H2D + xr_reduce_sharded + D2H"}
+               "api": "xr_reduce_host (C ABI: pinned host input, chunked H2D overlapped with the reduction)"
+               if world == 1 else "xr_reduce_sharded_host (C ABI: chunked H2D + local reduction + NCCL)",
+               "h2d_gbs_achieved": n * esz * args.e2e_steps / el / 1e9,
+               "pinned_h2d_gbs_measured": h2d,
+               "frac_of_pinned_h2d": n * esz * args.e2e_steps / el / 1e9 / h2d}
 
     cpu = cpu_omp = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         sample_n = min(n, 1 << 26)
+        model = cpu_model()
         rate, reps, el = oracle_rate(wl, host.numpy()[:sample_n], args.cpu_seconds)
-        cpu = {"value": rate, "unit": "elements/s", "cores": 1, "kind": "oracle",
+        cpu = {"value": rate, "unit": "elements/s", "cores": 1, "kind": "oracle", "cpu_model": model,
                "sample": f"{reps} x oracle over the first {sample_n} elements ({el:.1f} s, 1 thread)"}
         rate, reps, el, cores = openmp_rate(wl, host.numpy()[:sample_n], min(args.cpu_seconds, 3.0))
-        cpu_omp = {"value": rate, "unit": "elements/s", "cores": cores, "kind": "openmp",
+        cpu_omp = {"value": rate, "unit": "elements/s", "cores": cores, "kind": "openmp", "cpu_model": model,
                    "sample": f"{reps} x cpubase/omp.c over the first {sample_n} elements ({el:.1f} s, "
                              f"{cores} threads)"}
 
     if rank == 0:
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": ncu.get("traffic") if ncu else None,
+                "peak_source": peak_src,
+                # the metric's own unit: ncu dram__throughput % of peak for this
+                # kernel, from the committed capture named in ncu_source
+                "ncu_dram_pct": ncu.get("dram_pct") if ncu else None,
+                "ncu_source": ncu.get("source") if ncu else None,
+                "kernel": kernel_name,
+                "algorithmic_bytes_per_launch": alg_bytes,
+                "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)}
         line = {
             "metric": METRIC, "value": value, "unit": "elements/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": DTYPE_TAG[dtype],
             "data": "synthetic (seeded splitmix64 generator, datagen/)",
             "config": dict(workload_desc(wl, n, world, args.scaling), **({"exchange": exchange} if exchange else {})),
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "peak_source": peak_src,
-                         # context: the measured peak is a device COPY (read + write); a pure
-                         # read stream can exceed it, so also quote the nominal HGX figure
-                         "frac_of_nominal_7700": achieved / 7700.0,
-                         "kernel": kernel_name,
-                         "algorithmic_bytes_per_launch": alg_bytes,
-                         "kernel_ms_mean": kern_ms, "kernel_ms_min": min(per)},
+            "roofline": roof,
             "hbm_frac_of_peak": achieved / peak,
             "e2e": e2e,
             "gpu_launches": launches,
@@ -407,6 +524,8 @@ def run_gpu(args):
             "cpu_baseline": cpu,
             "cpu_baseline_openmp": cpu_omp,
         }
+        if multi is not None:
+            line["multi_gpu"] = multi
         print(json.dumps(line), flush=True)
     if comm is not None:
         comm.close()
@@ -417,6 +536,9 @@ def run_gpu(args):
 
 def main():
     args = parse()
+    rc = launch_ranks(args)
+    if rc is not None:
+        return rc
     if args.impl == "reference":
         return run_reference(args)
     return run_gpu(args)

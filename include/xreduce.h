@@ -117,13 +117,32 @@ int xr_out_count(const int64_t nest_dims[3], unsigned level_mask, int64_t* count
 /* Static string for a status code (never NULL). */
 const char* xr_strerror(int status);
 
-/* Same as xr_reduce but with HOST buffers: copies in (host, pinned or
- * pageable) to a library-owned device staging buffer in chunks along the gang
- * level, overlapping the copy of chunk c+1 with the reduction of chunk c, and
- * copies the result back into out (host).  Synchronous: returns after out is
- * written.  `stream` orders the work; NULL uses the legacy stream. */
+/* Same as xr_reduce but with HOST buffers (pinned or pageable; pinned gives
+ * the full PCIe rate).  The input is copied in bounded chunks (at most 32 MiB
+ * each, XR_HOST_CHUNK_BYTES overrides) through TWO library-owned device
+ * staging buffers on an internal copy stream, so the H2D copy of chunk c+1
+ * overlaps the reduction of chunk c on `stream`.  Chunks run along the
+ * outermost level whose single index fits in a chunk (earlier levels are
+ * iterated one index at a time); a chunk's outputs are one contiguous block of
+ * out.  When
+ * the chunk level or a level before it is REDUCED, several chunks share an
+ * output block: the first writes it (merging the caller's init), the later
+ * ones combine into it (their init is the block's current value) -- the gang
+ * tier across chunks, exact for integer / bitwise / logical / min / max and
+ * within C9 / C10 for fp + and *.  Staging is owned per (device, stream): the
+ * input buffers are 2 x min(chunk, input bytes), plus a device copy of the
+ * output (xr_out_count elements).  Synchronous: returns after out (host) is
+ * written; `stream` orders the work (NULL = legacy stream); concurrent calls
+ * on different streams use different staging.  Errors as xr_reduce. */
 int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                    const void* in_host, void* out_host, xr_stream_t stream);
+
+/* Host-only (no CUDA): the chunks xr_reduce_host would use with a chunk cap
+ * of cap_bytes.  Writes up to max_chunks rows of 6 int64 to out6: chunk dims
+ * n0, n1, n2, input offset (elements), output offset (elements), and 1 if the
+ * chunk is the first to write its output block.  *nchunks = total count. */
+int xr_host_chunks(const int64_t nest_dims[3], unsigned level_mask, int dtype, int64_t cap_bytes,
+                   int64_t max_chunks, int64_t* out6, int64_t* nchunks);
 
 /* Transform-reduce (the loop body before the reduction), two
  * inputs of the same nest (DEVICE, dtype-aligned, caller-owned):
@@ -276,8 +295,11 @@ int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,
  * must start with the initial field AND the neighbours' halo rows.  One step =
  * the fused sweep of the owned interior rows, then the halo rows of T2 are
  * exchanged with grouped ncclSend/ncclRecv and the residual is combined with
- * ncclAllReduce(max) of one fp64 into *residual (DEVICE) on every rank.  The
- * results are bit-identical to xr_heat_step on the whole grid. */
+ * ncclAllReduce(max) of one fp64 into *residual (DEVICE) on every rank (also
+ * at 1 rank).  The results are bit-identical to xr_heat_step on the whole
+ * grid.  With XR_FORCE_COLL set and 1 rank (tests), the rank exchanges its
+ * halos with itself: halo row 0 <- owned row 1, halo row n_local+1 <- owned
+ * row n_local (both halos are unused at the global boundary). */
 int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* T2,
                          double* residual, xr_comm_t comm, xr_stream_t stream);
 /* iters steps swapping T1/T2 (residuals: DEVICE, iters fp64). */
@@ -335,20 +357,41 @@ int xr_comm_destroy(xr_comm_t comm);
  * and combines the values in rank order -- ONE kernel, no NCCL launch, the same
  * bits on every rank.  Set up at xr_comm_init if every peer can be mapped;
  * otherwise (or when disabled) the NCCL collectives below are used.  The wait
- * is bounded: a rank that never arrives sets the status read by
- * xr_comm_query instead of hanging the GPU. */
+ * is bounded (20 s of %globaltimer; XR_EXCH_TIMEOUT_MS overrides): a rank
+ * whose peers never arrive leaves out UNCHANGED and sets a host-mapped status
+ * word, read by xr_comm_query without synchronising; while it is set, every
+ * fused xr_reduce_sharded call returns XR_ERR_NCCL.
+ * xr_comm_set_fused(comm, 0) switches this rank to the NCCL path (local, no
+ * communication).  xr_comm_set_fused(comm, 1) is COLLECTIVE (every rank calls
+ * it, nothing of the communicator in flight): it synchronises the device,
+ * re-aligns the mailbox epochs across ranks (NCCL max), clears the status word
+ * and enables the exchange; XR_ERR_UNSUPPORTED if a peer is not mapped. */
 int xr_comm_set_fused(xr_comm_t comm, int enable);
 int xr_comm_query(xr_comm_t comm, int* fused, int* status);
 
 /* Local xr_reduce on this rank's gang slice + ONE collective on `stream`
- * (or the fused exchange above). */
+ * (or the fused exchange above).  The collective runs at every world size,
+ * including a 1-rank communicator.  Errors: as xr_reduce, XR_ERR_NCCL for an
+ * NCCL failure or a timed-out fused exchange (see above). */
 int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
                       const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream);
+
+/* xr_reduce_sharded with HOST buffers: this rank's gang slice in_local_host
+ * (host, pinned for the full PCIe rate) goes through the chunked H2D pipeline
+ * of xr_reduce_host into a device partial, then the same collective as
+ * xr_reduce_sharded (NCCL; the fused exchange needs a single-launch local
+ * reduction and is not used here), and the GLOBAL result is copied to
+ * out_host (host; global_count elements, also the init when
+ * XR_INIT_FROM_OUT).  Synchronous.  Every rank calls it (NCCL rule). */
+int xr_reduce_sharded_host(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                           const void* in_local_host, void* out_host, xr_comm_t comm, xr_stream_t stream);
 
 /* Single-device simulation of the fused exchange: nranks concurrent kernels on
  * separate streams, each reducing shards[r] into outs[r] (1 element) with its
  * own mailbox -- the real publish / spin / combine protocol.  Synchronous.
- * XR_ERR_NCCL if a rank never arrived. */
+ * XR_ERR_NCCL if a rank never arrived (the waiting ranks leave their out
+ * unchanged).  Test hooks: XR_TEST_SIM_SKIP_RANK=r never launches rank r;
+ * XR_EXCH_TIMEOUT_MS bounds the wait (default 10 s here). */
 int xr_reduce_fused_sim(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
                         const void* const* shards, int nranks, void* const* outs);
 

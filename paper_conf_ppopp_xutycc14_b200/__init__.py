@@ -90,6 +90,7 @@ _SIGS = {
     "xr_out_count": (_c, [_i64p, _u, _i64p]),
     "xr_strerror": (ctypes.c_char_p, [_c]),
     "xr_reduce_host": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp]),
+    "xr_host_chunks": (_c, [_i64p, _u, _c, ctypes.c_int64, ctypes.c_int64, _i64p, _i64p]),
     "xr_plan_describe": (_c, [_c, _c, _i64p, _u, ctypes.c_uint64, _c, ctypes.POINTER(PlanInfo)]),
     "xr_reserve": (_c, [_c, _c, _i64p, _u, _vp]),
     "xr_shutdown": (_c, []),
@@ -101,6 +102,7 @@ _SIGS = {
     "xr_comm_init": (_c, [ctypes.POINTER(_vp), _c, _c, _vp, _c]),
     "xr_comm_destroy": (_c, [_vp]),
     "xr_reduce_sharded": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
+    "xr_reduce_sharded_host": (_c, [_c, _c, _i64p, _u, _vp, _vp, _vp, _vp]),
     "xr_reduce_sharded_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, _vp, _vp]),
     "xr_reduce_fused_sim": (_c, [_c, _c, _i64p, _u, ctypes.POINTER(_vp), _c, ctypes.POINTER(_vp)]),
     "xr_comm_set_fused": (_c, [_vp, _c]),
@@ -183,6 +185,19 @@ def xr_reduce_host(op, dtype, nest_dims, level_mask, in_host_ptr: int, out_host_
                    stream: int = 0) -> int:
     return _lib.xr_reduce_host(_op(op), _dt(dtype), _dims(nest_dims), mask_of(level_mask),
                                in_host_ptr or None, out_host_ptr or None, stream or None)
+
+
+def xr_host_chunks(nest_dims, level_mask, dtype, cap_bytes: int) -> list:
+    """The chunk schedule of xr_reduce_host (host only): a list of
+    (dims, in_off, out_off, first) tuples."""
+    n = ctypes.c_int64(0)
+    _check(_lib.xr_host_chunks(_dims(nest_dims), mask_of(level_mask), _dt(dtype), cap_bytes, 0, None,
+                               ctypes.byref(n)), "xr_host_chunks")
+    buf = (ctypes.c_int64 * (6 * max(n.value, 1)))()
+    _check(_lib.xr_host_chunks(_dims(nest_dims), mask_of(level_mask), _dt(dtype), cap_bytes, n.value,
+                               ctypes.cast(buf, _i64p), ctypes.byref(n)), "xr_host_chunks")
+    return [((buf[6 * k], buf[6 * k + 1], buf[6 * k + 2]), buf[6 * k + 3], buf[6 * k + 4], bool(buf[6 * k + 5]))
+            for k in range(n.value)]
 
 
 def xr_reserve(op, dtype, nest_dims, level_mask, stream: int = 0) -> int:
@@ -273,36 +288,67 @@ def _torch_dtypes():
     return _TORCH_DT
 
 
-def _stream_handle(stream=None) -> int:
+def _stream_handle(stream=None, device=None) -> int:
     import torch
-    s = stream if stream is not None else torch.cuda.current_stream()
+    s = stream if stream is not None else torch.cuda.current_stream(device)
     return int(s.cuda_stream)
 
 
+def _nest_of(x, nest):
+    """The (n0, n1, n2) view of tensor ``x``: ``nest`` if given (its product
+    must equal x.numel()), else x.shape with leading dimensions beyond the
+    last two flattened into n0 (and missing ones padded with 1 on the left)."""
+    if nest is None:
+        shp = [int(v) for v in x.shape]
+        if len(shp) > 3:
+            lead = 1
+            for v in shp[:-2]:
+                lead *= v
+            shp = [lead] + shp[-2:]
+        nest = [1] * (3 - len(shp)) + shp
+    nest = [int(v) for v in nest]
+    if len(nest) != 3 or any(v < 0 for v in nest):
+        raise ValueError(f"nest must be 3 non-negative extents, got {nest}")
+    if nest[0] * nest[1] * nest[2] != x.numel():
+        raise ValueError(f"nest {tuple(nest)} has {nest[0] * nest[1] * nest[2]} elements but the tensor has "
+                         f"{x.numel()}")
+    return nest
+
+
+def _check_out(out, x, count: int):
+    if out.dtype != x.dtype:
+        raise ValueError(f"out dtype {out.dtype} differs from the input's {x.dtype}")
+    if out.device != x.device:
+        raise ValueError(f"out is on {out.device}, the input on {x.device}")
+    if out.numel() < count or not out.is_contiguous():
+        raise ValueError(f"out must be contiguous with at least {count} elements (has {out.numel()})")
+
+
 def reduce(x, op="+", levels="gwv", nest=None, out=None, init=None, stream=None):
-    """Reduce CUDA tensor ``x`` (viewed as nest ``(n0, n1, n2)``, default: x.shape
-    padded to 3 dims on the left) over ``levels``; returns the compact output
-    tensor (shape = the kept extents)."""
+    """Reduce CUDA tensor ``x`` (viewed as nest ``(n0, n1, n2)``; default:
+    x.shape, leading dims beyond 3 flattened into n0) over ``levels``;
+    returns the compact output tensor (shape = the kept extents).  Runs on
+    x's device, on ``stream`` or that device's current stream."""
     import torch
     if not x.is_cuda:
         raise ValueError("xreduce.reduce needs a CUDA tensor (no CPU fallback)")
+    if x.dtype not in _torch_dtypes():
+        raise ValueError(f"unsupported dtype {x.dtype} (int32, int64, float32, float64)")
     x = x.contiguous()
-    if nest is None:
-        shp = list(x.shape)[-3:]
-        nest = [1] * (3 - len(shp)) + shp
-    nest = [int(v) for v in nest]
+    nest = _nest_of(x, nest)
     mask = mask_of(levels)
     dt = _torch_dtypes()[x.dtype]
     kept = [nest[d] for d in range(3) if not (mask >> d) & 1]
     count = xr_out_count(nest, mask)
-    if out is None:
-        out = torch.empty(kept if kept else [1], dtype=x.dtype, device=x.device)
-    if init is not None:
-        out.copy_(torch.as_tensor(init, dtype=x.dtype, device=x.device).reshape(out.shape))
-        mask |= INIT_FROM_OUT
-    assert out.numel() == count and out.is_contiguous()
-    _check(xr_reduce(_op(op), dt, nest, mask, x.data_ptr(), out.data_ptr(), _stream_handle(stream)),
-           "xr_reduce")
+    with torch.cuda.device(x.device):
+        if out is None:
+            out = torch.empty(kept if kept else [1], dtype=x.dtype, device=x.device)
+        _check_out(out, x, count)
+        if init is not None:
+            out.copy_(torch.as_tensor(init, dtype=x.dtype, device=x.device).reshape(out.shape))
+            mask |= INIT_FROM_OUT
+        _check(xr_reduce(_op(op), dt, nest, mask, x.data_ptr(), out.data_ptr(), _stream_handle(stream, x.device)),
+               "xr_reduce")
     return out
 
 
@@ -355,18 +401,22 @@ def reduce_sharded(x_local, comm: Comm, op="+", levels="gwv", nest_local=None, o
     """Gang-sharded reduction: every rank passes its contiguous gang slice;
     returns the GLOBAL result on every rank (include/xreduce.h)."""
     import torch
+    if not x_local.is_cuda:
+        raise ValueError("xreduce.reduce_sharded needs a CUDA tensor (no CPU fallback)")
+    if x_local.dtype not in _torch_dtypes():
+        raise ValueError(f"unsupported dtype {x_local.dtype} (int32, int64, float32, float64)")
     x_local = x_local.contiguous()
-    if nest_local is None:
-        shp = list(x_local.shape)[-3:]
-        nest_local = [1] * (3 - len(shp)) + shp
+    nest_local = _nest_of(x_local, nest_local)
     mask = mask_of(levels)
     info = xr_shard_plan(op, _torch_dtypes()[x_local.dtype], nest_local, mask, comm.nranks, comm.rank)
-    if out is None:
-        out = torch.empty(max(info["global_count"], 1), dtype=x_local.dtype, device=x_local.device)
-    if init is not None:
-        out.copy_(torch.as_tensor(init, dtype=x_local.dtype, device=out.device).reshape(out.shape))
-        mask |= INIT_FROM_OUT
-    _check(_lib.xr_reduce_sharded(_op(op), _torch_dtypes()[x_local.dtype], _dims(nest_local), mask,
-                                  x_local.data_ptr(), out.data_ptr(), comm.handle,
-                                  _stream_handle(stream)), "xr_reduce_sharded")
+    with torch.cuda.device(x_local.device):
+        if out is None:
+            out = torch.empty(max(info["global_count"], 1), dtype=x_local.dtype, device=x_local.device)
+        _check_out(out, x_local, info["global_count"])
+        if init is not None:
+            out.copy_(torch.as_tensor(init, dtype=x_local.dtype, device=out.device).reshape(out.shape))
+            mask |= INIT_FROM_OUT
+        _check(_lib.xr_reduce_sharded(_op(op), _torch_dtypes()[x_local.dtype], _dims(nest_local), mask,
+                                      x_local.data_ptr(), out.data_ptr(), comm.handle,
+                                      _stream_handle(stream, x_local.device)), "xr_reduce_sharded")
     return out

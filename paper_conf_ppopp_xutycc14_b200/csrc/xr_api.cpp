@@ -1,9 +1,12 @@
 // xr_api.cpp -- the C ABI (include/xreduce.h): validation, workspace, dispatch.
 // Validation never touches CUDA, so every status path is testable on a CPU
 // machine (tests/test_abi.py).
+#include <algorithm>
 #include <atomic>
 #include <cstring>
+#include <cstdlib>
 #include <map>
+#include <memory>
 #include <mutex>
 #include <utility>
 #include <vector>
@@ -164,8 +167,18 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   p.rkr.in = in; p.rkr.out = out; p.rkr.partials = w.partials; p.rkr.tickets = w.tickets;
   p.rkr.sched = sched; p.rkr.init_from_out = ifo;
   if (p.kernel == K_COLTMA && !make_col_tmap(&p.tmap, dtype, in, p.col.B, p.col.R, p.col.K)) {
-    // no tensor-map support: re-plan without TMA (same workspace bound or smaller)
-    return XR_ERR_CUDA;
+    // no tensor-map support (driver entry point or encode failed): re-plan
+    // onto the register column kernels and launch those instead
+    Plan q;
+    make_plan(op, dtype, dims, mask & 7u, (uint64_t)(uintptr_t)in, sms, &q, false, 0, false, /*no_tma=*/true);
+    q.seg = p.seg;  // keep the exchange fields (unused by column plans)
+    p = q;
+    const int64_t words = (p.tickets + 1) & ~int64_t(1);
+    if ((st = ensure_ws(w, p.ws_bytes, words + (p.sched ? 4 : 0), stream))) return st;
+    sched = reinterpret_cast<unsigned long long*>(w.tickets + words);
+    p.col.in = in; p.col.out = out; p.col.partials = w.partials; p.col.tickets = w.tickets;
+    p.col.init_from_out = ifo; p.col.sched = sched;
+    p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
   }
   cudaError_t e = launch_dtype(op, dtype, p, sms, stream);
   if (e != cudaSuccess) {
@@ -177,27 +190,228 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
 }
 
 // ---------------------------------------------------------------- host-buffer path
+// xr_reduce_host: the input is copied in bounded chunks through two device
+// staging buffers on a copy stream, overlapping the H2D copy of chunk c+1 with
+// the reduction of chunk c on the caller's stream (include/xreduce.h).  One
+// staging context per (device, stream); the call is synchronous and holds the
+// context's mutex throughout, so concurrent calls on different streams never
+// share buffers and calls on one stream serialise.
+constexpr size_t kHostChunkBytes = size_t(32) << 20;  // per staging buffer
 struct Staging {
-  void* in = nullptr;
+  std::mutex mu;
+  void* in[2] = {nullptr, nullptr};
   size_t in_bytes = 0;
   void* out = nullptr;
   size_t out_bytes = 0;
+  cudaStream_t copy = nullptr;
+  cudaEvent_t copied[2] = {nullptr, nullptr};
+  cudaEvent_t consumed[2] = {nullptr, nullptr};
 };
-static std::map<int, Staging> g_stage;
+static std::map<std::pair<int, uintptr_t>, std::unique_ptr<Staging>> g_stage;  // guarded by g_mu
 
-static int grow(void** p, size_t* have, size_t need) {
-  if (need <= *have) return XR_OK;
-  if (*p) { cudaDeviceSynchronize(); cudaFree(*p); }
-  *p = nullptr;
-  *have = 0;
-  if (cudaMalloc(p, need) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
-  *have = need;
+static void free_staging(Staging& sg) {
+  for (int b = 0; b < 2; ++b) {
+    if (sg.in[b]) cudaFree(sg.in[b]);
+    sg.in[b] = nullptr;
+    if (sg.copied[b]) cudaEventDestroy(sg.copied[b]);
+    if (sg.consumed[b]) cudaEventDestroy(sg.consumed[b]);
+    sg.copied[b] = sg.consumed[b] = nullptr;
+  }
+  sg.in_bytes = 0;
+  if (sg.out) cudaFree(sg.out);
+  sg.out = nullptr;
+  sg.out_bytes = 0;
+  if (sg.copy) cudaStreamDestroy(sg.copy);
+  sg.copy = nullptr;
+}
+
+// Buffers and streams for a call needing `chunk` bytes per input buffer and
+// `obytes` of output (caller holds sg.mu; no work of this context is in flight).
+static int prepare_staging(Staging& sg, size_t chunk, size_t obytes) {
+  if (!sg.copy) {
+    if (cudaStreamCreateWithFlags(&sg.copy, cudaStreamNonBlocking) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+    for (int b = 0; b < 2; ++b)
+      if (cudaEventCreateWithFlags(&sg.copied[b], cudaEventDisableTiming) != cudaSuccess ||
+          cudaEventCreateWithFlags(&sg.consumed[b], cudaEventDisableTiming) != cudaSuccess) {
+        cudaGetLastError();
+        return XR_ERR_CUDA;
+      }
+  }
+  if (chunk > sg.in_bytes) {
+    for (int b = 0; b < 2; ++b) {
+      if (sg.in[b]) cudaFree(sg.in[b]);
+      sg.in[b] = nullptr;
+    }
+    sg.in_bytes = 0;
+    for (int b = 0; b < 2; ++b)
+      if (cudaMalloc(&sg.in[b], chunk) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+    sg.in_bytes = chunk;
+  }
+  if (obytes > sg.out_bytes) {
+    if (sg.out) cudaFree(sg.out);
+    sg.out = nullptr;
+    sg.out_bytes = 0;
+    if (cudaMalloc(&sg.out, obytes) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+    sg.out_bytes = obytes;
+  }
   return XR_OK;
+}
+
+// One chunk of the nest: index prefix fixed on the levels before `lvl`, the
+// range [a, a + ext) on level `lvl`, full extents after it.
+struct HostChunk {
+  int64_t dims[3];
+  int64_t in_off;    // elements
+  int64_t out_off;   // elements: the chunk's outputs are one contiguous block
+  bool first;        // no earlier chunk wrote this output block
+};
+
+// Chunks of at most `cap` bytes in input order (exposed for the CPU tests
+// through xr_host_chunks).  The chunk level is the outermost level whose
+// single index fits in `cap`; a chunk's outputs are contiguous because every
+// level after the chunk level is complete.  An output block is written first
+// by the chunk whose indices on every REDUCED level up to the chunk level are
+// 0; later chunks of the same block accumulate into it (init from out).
+template <typename F>
+static void for_each_chunk(const int64_t n[3], unsigned mask, int size, int64_t cap, F f) {
+  int64_t row[3];  // bytes of one index of level d
+  row[2] = size;
+  row[1] = row[2] * n[2];
+  row[0] = row[1] * n[1];
+  int lvl = 2;
+  for (int d = 0; d < 3; ++d)
+    if (row[d] <= cap) { lvl = d; break; }
+  const int64_t per = std::max<int64_t>(1, cap / row[lvl]);
+  const int64_t istride[3] = {n[1] * n[2], n[2], 1};
+  int64_t ostride[3];
+  int64_t acc = 1;
+  for (int d = 2; d >= 0; --d) {
+    ostride[d] = acc;
+    if (!((mask >> d) & 1u)) acc *= n[d];
+  }
+  const int64_t p0 = lvl > 0 ? n[0] : 1, p1 = lvl > 1 ? n[1] : 1;
+  for (int64_t i0 = 0; i0 < p0; ++i0)
+    for (int64_t i1 = 0; i1 < p1; ++i1)
+      for (int64_t a = 0; a < n[lvl]; a += per) {
+        HostChunk c;
+        const int64_t idx[3] = {lvl == 0 ? a : i0, lvl == 1 ? a : (lvl > 1 ? i1 : 0), lvl == 2 ? a : 0};
+        c.first = true;
+        c.in_off = 0;
+        c.out_off = 0;
+        for (int d = 0; d < 3; ++d) {
+          c.dims[d] = d < lvl ? 1 : d == lvl ? std::min(per, n[lvl] - a) : n[d];
+          if (d > lvl) continue;
+          c.in_off += idx[d] * istride[d];
+          if ((mask >> d) & 1u) c.first = c.first && idx[d] == 0;
+          else c.out_off += idx[d] * ostride[d];
+        }
+        f(c);
+      }
+}
+
+static int64_t host_chunk_cap() {
+  const char* e = std::getenv("XR_HOST_CHUNK_BYTES");  // test / tuning override
+  const int64_t v = e ? std::atoll(e) : (int64_t)kHostChunkBytes;
+  return std::max<int64_t>(v, 16);
+}
+
+static size_t chunk_bytes_for(int64_t total_bytes) {
+  return (size_t)std::max<int64_t>(std::min<int64_t>(total_bytes, host_chunk_cap()), 16);
+}
+
+static int staging_for(xr_stream_t stream, Staging** out) {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  std::lock_guard<std::mutex> lock(g_mu);
+  auto& slot = g_stage[{dev, (uintptr_t)stream}];
+  if (!slot) slot.reset(new Staging());
+  *out = slot.get();
+  return XR_OK;
+}
+
+// The chunked H2D + reduce pipeline into the DEVICE output dout (which holds
+// the init when mask has XR_INIT_FROM_OUT).  Caller holds sg.mu and has
+// prepared the input buffers; enqueues only (the caller synchronises).
+static int pipeline_locked(Staging& sg, int op, int dtype, const int64_t* dims, unsigned mask,
+                           const void* in_host, char* dout, cudaStream_t s) {
+  const int size = dtype_size(dtype);
+  const int64_t total = dims[0] * dims[1] * dims[2];
+  const bool ifo = (mask & XR_INIT_FROM_OUT) != 0;
+  const unsigned base = mask & 7u;
+  if (total == 0) return reduce_device(op, dtype, dims, mask, nullptr, dout, s);  // out = init (C17)
+  // the copy stream starts after the caller's prior work on `stream`, and
+  // never overwrites a buffer before the reduction reading it (chunk c-2)
+  if (cudaEventRecord(sg.consumed[0], s) != cudaSuccess || cudaStreamWaitEvent(sg.copy, sg.consumed[0], 0) != cudaSuccess) {
+    cudaGetLastError();
+    return XR_ERR_CUDA;
+  }
+  int st = XR_OK;
+  int64_t c = 0;
+  for_each_chunk(dims, base, size, host_chunk_cap(), [&](const HostChunk& ch) {
+    if (st) return;
+    const int b = (int)(c & 1);
+    const int64_t bytes = ch.dims[0] * ch.dims[1] * ch.dims[2] * size;
+    if ((c >= 2 && cudaStreamWaitEvent(sg.copy, sg.consumed[b], 0) != cudaSuccess) ||
+        cudaMemcpyAsync(sg.in[b], static_cast<const char*>(in_host) + ch.in_off * size, (size_t)bytes,
+                        cudaMemcpyHostToDevice, sg.copy) != cudaSuccess ||
+        cudaEventRecord(sg.copied[b], sg.copy) != cudaSuccess || cudaStreamWaitEvent(s, sg.copied[b], 0) != cudaSuccess) {
+      cudaGetLastError();
+      st = XR_ERR_CUDA;
+      return;
+    }
+    const unsigned m = base | ((!ch.first || ifo) ? XR_INIT_FROM_OUT : 0u);
+    st = reduce_device(op, dtype, ch.dims, m, sg.in[b], dout + ch.out_off * size, s);
+    if (!st && cudaEventRecord(sg.consumed[b], s) != cudaSuccess) { cudaGetLastError(); st = XR_ERR_CUDA; }
+    ++c;
+  });
+  return st;
+}
+
+// used by xr_comm.cpp (xr_reduce_sharded_host): the pipeline into a caller's
+// device buffer; synchronous.
+int reduce_host_into(int op, int dtype, const int64_t* dims, unsigned mask, const void* in_host, void* out_dev,
+                     cudaStream_t s) {
+  int64_t total = 0, count = 0;
+  int st = validate(op, dtype, dims, mask, &total, &count);
+  if (st) return st;
+  if (count == 0) return XR_OK;
+  if (!out_dev || (total > 0 && !in_host)) return XR_ERR_INVALID;
+  Staging* sgp = nullptr;
+  if ((st = staging_for((xr_stream_t)s, &sgp))) return st;
+  Staging& sg = *sgp;
+  std::lock_guard<std::mutex> call_lock(sg.mu);
+  if ((st = prepare_staging(sg, chunk_bytes_for(total * dtype_size(dtype)), 0))) return st;
+  st = pipeline_locked(sg, op, dtype, dims, mask, in_host, static_cast<char*>(out_dev), s);
+  const cudaError_t e1 = cudaStreamSynchronize(sg.copy);
+  const cudaError_t e2 = cudaStreamSynchronize(s);
+  if (!st && (e1 != cudaSuccess || e2 != cudaSuccess)) st = XR_ERR_CUDA;
+  if (st) cudaGetLastError();
+  return st;
 }
 
 }  // namespace xr
 
 using namespace xr;
+
+extern "C" int xr_host_chunks(const int64_t nest_dims[3], unsigned level_mask, int dtype, int64_t cap_bytes,
+                              int64_t max_chunks, int64_t* out6, int64_t* nchunks) {
+  int64_t total = 0, count = 0;
+  int st = validate(XR_OP_ADD, dtype, nest_dims, level_mask, &total, &count);
+  if (st) return st;
+  if (!nchunks || cap_bytes < 1 || max_chunks < 0 || (max_chunks > 0 && !out6)) return XR_ERR_INVALID;
+  int64_t k = 0;
+  if (total > 0)
+    for_each_chunk(nest_dims, level_mask & 7u, dtype_size(dtype), cap_bytes, [&](const HostChunk& c) {
+      if (k < max_chunks) {
+        int64_t* o = out6 + 6 * k;
+        o[0] = c.dims[0]; o[1] = c.dims[1]; o[2] = c.dims[2];
+        o[3] = c.in_off; o[4] = c.out_off; o[5] = c.first ? 1 : 0;
+      }
+      ++k;
+    });
+  *nchunks = k;
+  return XR_OK;
+}
 
 extern "C" {
 
@@ -282,8 +496,8 @@ int xr_shutdown(void) {
   }
   g_ws.clear();
   for (auto& kv : g_stage) {
-    if (kv.second.in) cudaFree(kv.second.in);
-    if (kv.second.out) cudaFree(kv.second.out);
+    std::lock_guard<std::mutex> sl(kv.second->mu);
+    free_staging(*kv.second);
   }
   g_stage.clear();
   cudaGetLastError();
@@ -300,30 +514,29 @@ int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level
   if (count == 0) return XR_OK;
   if (!out_host || (total > 0 && !in_host)) return XR_ERR_INVALID;
   const int size = dtype_size(dtype);
-  int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
-  void* din;
-  void* dout;
-  {
-    std::lock_guard<std::mutex> lock(g_mu);
-    Staging& sg = g_stage[dev];
-    if ((st = grow(&sg.in, &sg.in_bytes, (size_t)std::max<int64_t>(total * size, 16)))) return st;
-    if ((st = grow(&sg.out, &sg.out_bytes, (size_t)count * size))) return st;
-    din = sg.in;
-    dout = sg.out;
-  }
   cudaStream_t s = (cudaStream_t)stream;
+  Staging* sgp = nullptr;
+  if ((st = staging_for(stream, &sgp))) return st;
+  Staging& sg = *sgp;
+  std::lock_guard<std::mutex> call_lock(sg.mu);  // held for the whole (synchronous) call
+  if ((st = prepare_staging(sg, chunk_bytes_for(total * size), (size_t)count * size))) return st;
+  char* dout = static_cast<char*>(sg.out);
   if ((level_mask & XR_INIT_FROM_OUT) &&
-      cudaMemcpyAsync(dout, out_host, (size_t)count * size, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      cudaMemcpyAsync(dout, out_host, (size_t)count * size, cudaMemcpyHostToDevice, s) != cudaSuccess) {
+    cudaGetLastError();
     return XR_ERR_CUDA;
-  if (total > 0 && cudaMemcpyAsync(din, in_host, (size_t)total * size, cudaMemcpyHostToDevice, s) != cudaSuccess)
-    return XR_ERR_CUDA;
-  st = reduce_device(op, dtype, nest_dims, level_mask, din, dout, s);
-  if (st) return st;
-  if (cudaMemcpyAsync(out_host, dout, (size_t)count * size, cudaMemcpyDeviceToHost, s) != cudaSuccess)
-    return XR_ERR_CUDA;
-  if (cudaStreamSynchronize(s) != cudaSuccess) return XR_ERR_CUDA;
-  return XR_OK;
+  }
+  st = pipeline_locked(sg, op, dtype, nest_dims, level_mask, in_host, dout, s);
+  if (!st && cudaMemcpyAsync(out_host, dout, (size_t)count * size, cudaMemcpyDeviceToHost, s) != cudaSuccess) {
+    cudaGetLastError();
+    st = XR_ERR_CUDA;
+  }
+  // both streams drain before the buffers can be reused (also on errors)
+  const cudaError_t e1 = cudaStreamSynchronize(sg.copy);
+  const cudaError_t e2 = cudaStreamSynchronize(s);
+  if (!st && (e1 != cudaSuccess || e2 != cudaSuccess)) st = XR_ERR_CUDA;
+  if (st) cudaGetLastError();
+  return st;
 }
 
 // ------------------------------------------------------------ sharding plan
@@ -436,14 +649,23 @@ int xr_reduce_fused_sim(int op, int dtype, const int64_t local_dims[3], unsigned
   cudaDeviceSynchronize();
   cudaMemcpy(outs[0], &saved, dtype_size(dtype), cudaMemcpyHostToDevice);
   // every "rank" is a concurrent kernel on its own stream; the last CTA of
-  // each spins on its mailbox until all the others published (real protocol)
+  // each spins on its mailbox until all the others published (real protocol).
+  // XR_TEST_SIM_SKIP_RANK=r (tests): rank r never launches, so the others
+  // must time out (XR_EXCH_TIMEOUT_MS), leave their out unchanged and report.
+  const char* skip_env = std::getenv("XR_TEST_SIM_SKIP_RANK");
+  const int skip = skip_env ? std::atoi(skip_env) : -1;
+  const char* to_env = std::getenv("XR_EXCH_TIMEOUT_MS");
+  const unsigned long long timeout_ns =
+      (unsigned long long)std::max(1ll, to_env ? std::atoll(to_env) : 10000ll) * 1000000ull;
   for (int r = 0; r < nranks && !st; ++r) {
+    if (r == skip) continue;
     ExchArgs x{};
     x.mine = mb + (size_t)r * kMailboxWords;
     for (int p = 0; p < nranks; ++p) x.peers[p] = mb + (size_t)p * kMailboxWords;
     x.nranks = nranks;
     x.rank = r;
     x.epoch = 1;
+    x.timeout_ns = timeout_ns;
     x.status = status;
     xr_shard_info info;
     xr_shard_plan(op, dtype, local_dims, level_mask, nranks, r, &info);

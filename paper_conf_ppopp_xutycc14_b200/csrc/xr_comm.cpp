@@ -7,6 +7,8 @@
 // (blocking across GPUs; the paper notes blocking and window sliding are
 // equivalent for gang partial reduction, @25998-26464), then ONE collective
 // over NVLink/NVSwitch combines them (xr_shard_plan decides which).
+#include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 #include <nccl.h>
@@ -21,6 +23,8 @@ cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t
 int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* je);
 int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
                    double* residual, cudaStream_t s);
+int reduce_host_into(int op, int dtype, const int64_t* dims, unsigned mask, const void* in_host, void* out_dev,
+                     cudaStream_t s);
 }  // namespace xr
 
 using xr::kMaxRanks;
@@ -32,25 +36,41 @@ struct xr_comm_s {
   int nranks = 0, rank = 0, device = 0;
   void* scratch = nullptr;  // allgather buffers for & | ^
   size_t scratch_bytes = 0;
+  void* hout = nullptr;     // device copy of the output of xr_reduce_sharded_host
+  size_t hout_bytes = 0;
   // fused exchange (peer mailboxes over NVLink via CUDA IPC)
   bool fused = false;                         // set up and enabled
   unsigned long long* mailbox = nullptr;      // mine
   unsigned long long* peers[kMaxRanks] = {};  // every rank's mailbox, mapped into this process
-  int* status = nullptr;
+  int* status = nullptr;        // host-mapped pinned word (device pointer below)
+  int* status_dev = nullptr;
   unsigned long long epoch = 0;
+  unsigned long long timeout_ns = 0;
 };
+
+// Wait bound of the fused exchange: a peer later than this is reported (the
+// host-mapped status word) instead of hanging the GPU.  XR_EXCH_TIMEOUT_MS
+// overrides (tests).
+static unsigned long long exch_timeout_ns() {
+  const char* e = std::getenv("XR_EXCH_TIMEOUT_MS");
+  const long long ms = e ? std::atoll(e) : 20000;
+  return (unsigned long long)std::max(1ll, ms) * 1000000ull;
+}
 
 // Allocate this rank's mailbox, all-gather the CUDA IPC handles with NCCL and
 // map every peer's mailbox.  Any failure leaves the communicator on NCCL.
 static void setup_fused(xr_comm_s* c) {
   if (c->nranks > kMaxRanks) return;
   const size_t bytes = kMailboxWords * sizeof(unsigned long long);
-  if (cudaMalloc(&c->mailbox, bytes) != cudaSuccess || cudaMalloc(&c->status, sizeof(int)) != cudaSuccess) {
+  if (cudaMalloc(&c->mailbox, bytes) != cudaSuccess ||
+      cudaHostAlloc(reinterpret_cast<void**>(&c->status), sizeof(int), cudaHostAllocMapped) != cudaSuccess ||
+      cudaHostGetDevicePointer(reinterpret_cast<void**>(&c->status_dev), c->status, 0) != cudaSuccess) {
     cudaGetLastError();
     return;
   }
   cudaMemset(c->mailbox, 0, bytes);
-  cudaMemset(c->status, 0, sizeof(int));
+  *reinterpret_cast<volatile int*>(c->status) = 0;
+  c->timeout_ns = exch_timeout_ns();
   c->peers[c->rank] = c->mailbox;
   if (c->nranks > 1) {
     cudaIpcMemHandle_t h;
@@ -135,27 +155,45 @@ int xr_comm_init(xr_comm_t* comm, int nranks, int rank, const void* id128, int d
   return XR_OK;
 }
 
+static int read_status(const xr_comm_s* c) {
+  return c->status ? *reinterpret_cast<volatile const int*>(c->status) : 0;
+}
+
 int xr_comm_set_fused(xr_comm_t comm, int enable) {
   if (!comm) return XR_ERR_INVALID;
-  if (enable && !comm->mailbox) return XR_ERR_UNSUPPORTED;
-  if (enable) {  // re-check that every peer is mapped
-    for (int p = 0; p < comm->nranks; ++p)
-      if (!comm->peers[p]) return XR_ERR_UNSUPPORTED;
+  if (!enable) {
+    comm->fused = false;
+    return XR_OK;
   }
-  comm->fused = enable != 0;
+  if (!comm->mailbox || !comm->status) return XR_ERR_UNSUPPORTED;
+  for (int p = 0; p < comm->nranks; ++p)  // every peer mapped
+    if (!comm->peers[p]) return XR_ERR_UNSUPPORTED;
+  // Collective: re-synchronise the mailbox epochs (a timed-out exchange can
+  // leave ranks at different epochs) and clear the status word.  Every rank
+  // calls this; nothing of this communicator may be in flight.
+  if (cudaSetDevice(comm->device) != cudaSuccess || cudaDeviceSynchronize() != cudaSuccess) {
+    cudaGetLastError();
+    return XR_ERR_CUDA;
+  }
+  unsigned long long* d = nullptr;
+  if (cudaMalloc(&d, sizeof *d) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+  unsigned long long e = comm->epoch;
+  int st = XR_OK;
+  if (cudaMemcpy(d, &e, sizeof e, cudaMemcpyHostToDevice) != cudaSuccess) st = XR_ERR_CUDA;
+  else if (ncclAllReduce(d, d, 1, ncclUint64, ncclMax, comm->nccl, 0) != ncclSuccess) st = XR_ERR_NCCL;
+  else if (cudaMemcpy(&e, d, sizeof e, cudaMemcpyDeviceToHost) != cudaSuccess) st = XR_ERR_CUDA;
+  cudaFree(d);
+  if (st) { cudaGetLastError(); return st; }
+  comm->epoch = e;
+  *reinterpret_cast<volatile int*>(comm->status) = 0;
+  comm->fused = true;
   return XR_OK;
 }
 
 int xr_comm_query(xr_comm_t comm, int* fused, int* status) {
   if (!comm) return XR_ERR_INVALID;
   if (fused) *fused = comm->fused ? 1 : 0;
-  if (status) {
-    *status = 0;
-    if (comm->status && cudaMemcpy(status, comm->status, sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess) {
-      cudaGetLastError();
-      return XR_ERR_CUDA;
-    }
-  }
+  if (status) *status = read_status(comm);  // host-mapped: no device synchronisation
   return XR_OK;
 }
 
@@ -165,22 +203,29 @@ int xr_comm_destroy(xr_comm_t comm) {
   for (int p = 0; p < comm->nranks && p < kMaxRanks; ++p)
     if (p != comm->rank && comm->peers[p]) cudaIpcCloseMemHandle(comm->peers[p]);
   if (comm->mailbox) cudaFree(comm->mailbox);
-  if (comm->status) cudaFree(comm->status);
+  if (comm->status) cudaFreeHost(comm->status);
   if (comm->scratch) cudaFree(comm->scratch);
+  if (comm->hout) cudaFree(comm->hout);
   if (comm->nccl && ncclCommDestroy(comm->nccl) != ncclSuccess) st = XR_ERR_NCCL;
   delete comm;
   return st;
 }
 
-int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
-                      const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream) {
-  if (!comm) return XR_ERR_INVALID;
+}  // extern "C"
+
+// The sharded protocol around a local reduction `local(mask, dst)` that writes
+// this rank's xr_out_count(local_dims) results to device memory dst (merging
+// dst as init when mask has XR_INIT_FROM_OUT).  fused_local: the same
+// reduction with the fused NVLink exchange (nullptr when the caller's local
+// reduction cannot host it).
+template <typename Local, typename FusedLocal>
+static int sharded_impl(int op, int dtype, const int64_t local_dims[3], unsigned level_mask, void* out,
+                        xr_comm_t comm, cudaStream_t s, Local local, FusedLocal* fused_local) {
   xr_shard_info info;
   int st = xr_shard_plan(op, dtype, local_dims, level_mask, comm->nranks, comm->rank, &info);
   if (st) return st;
   if (info.global_count == 0) return XR_OK;
   if (!out) return XR_ERR_INVALID;
-  cudaStream_t s = (cudaStream_t)stream;
   const int size = dtype_size(dtype);
   const unsigned base = (level_mask & 7u) | (info.local_init_from_out ? XR_INIT_FROM_OUT : 0u);
   char* mine = (char*)out + info.out_offset * size;
@@ -195,20 +240,23 @@ int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned l
       if (cudaMalloc(&comm->scratch, need) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
       comm->scratch_bytes = need;
     }
-    char* local = (char*)comm->scratch;
-    char* gathered = local + (size_t)info.local_count * size;
+    char* lbuf = (char*)comm->scratch;
+    char* gathered = lbuf + (size_t)info.local_count * size;
     if (info.local_init_from_out &&
-        cudaMemcpyAsync(local, out, (size_t)info.local_count * size, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
+        cudaMemcpyAsync(lbuf, out, (size_t)info.local_count * size, cudaMemcpyDeviceToDevice, s) != cudaSuccess)
       return XR_ERR_CUDA;
-    if ((st = reduce_device_checked(op, dtype, local_dims, base, in_local, local, s))) return st;
-    if (ncclAllGather(local, gathered, (size_t)info.local_count, nccl_type(dtype), comm->nccl, s) != ncclSuccess)
+    if ((st = local(base, lbuf))) return st;
+    if (ncclAllGather(lbuf, gathered, (size_t)info.local_count, nccl_type(dtype), comm->nccl, s) != ncclSuccess)
       return XR_ERR_NCCL;
     if (gather_combine(op, dtype, gathered, comm->nranks, info.local_count, out, s) != cudaSuccess)
       return XR_ERR_CUDA;
     return XR_OK;
   }
 
-  if (comm->fused && (level_mask & XR_GANG) && info.global_count == 1) {
+  if (fused_local && comm->fused && (level_mask & XR_GANG) && info.global_count == 1) {
+    // a previous fused exchange timed out: the mailbox epochs may disagree
+    // across ranks, so refuse until xr_comm_set_fused re-synchronises them
+    if (read_status(comm)) return XR_ERR_NCCL;
     // one kernel: local reduction + peer-mailbox exchange over NVLink
     ExchArgs x{};
     x.mine = comm->mailbox;
@@ -216,13 +264,17 @@ int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned l
     x.nranks = comm->nranks;
     x.rank = comm->rank;
     x.epoch = ++comm->epoch;
-    x.status = comm->status;
-    st = reduce_device_checked(op, dtype, local_dims, base, in_local, mine, s, &x);
+    x.timeout_ns = comm->timeout_ns;
+    x.status = comm->status_dev;
+    st = (*fused_local)(base, mine, &x);
+    if (st == XR_OK) return XR_OK;
+    --comm->epoch;  // nothing was launched: the epoch stays in step with the peers
     if (st != XR_ERR_UNSUPPORTED) return st;
-    --comm->epoch;  // this plan cannot host the exchange: NCCL below
+    // this plan cannot host the exchange: NCCL below
   }
-  if ((st = reduce_device_checked(op, dtype, local_dims, base, in_local, mine, s))) return st;
-  if (comm->nranks == 1) return XR_OK;
+  if ((st = local(base, mine))) return st;
+  // the collective runs at every world size (a 1-rank communicator executes
+  // the same NCCL call, so its op / dtype mapping is exercised on one GPU)
   if (info.collective == XR_COLL_ALLREDUCE) {
     if (ncclAllReduce(out, out, (size_t)info.global_count, nccl_type(dtype), (ncclRedOp_t)info.nccl_op,
                       comm->nccl, s) != ncclSuccess)
@@ -235,6 +287,55 @@ int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned l
   return XR_OK;
 }
 
+extern "C" {
+
+int xr_reduce_sharded(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                      const void* in_local, void* out, xr_comm_t comm, xr_stream_t stream) {
+  if (!comm) return XR_ERR_INVALID;
+  cudaStream_t s = (cudaStream_t)stream;
+  auto local = [&](unsigned m, void* dst) { return reduce_device_checked(op, dtype, local_dims, m, in_local, dst, s); };
+  auto fused = [&](unsigned m, void* dst, const ExchArgs* x) {
+    return reduce_device_checked(op, dtype, local_dims, m, in_local, dst, s, x);
+  };
+  return sharded_impl(op, dtype, local_dims, level_mask, out, comm, s, local, &fused);
+}
+
+int xr_reduce_sharded_host(int op, int dtype, const int64_t local_dims[3], unsigned level_mask,
+                           const void* in_local_host, void* out_host, xr_comm_t comm, xr_stream_t stream) {
+  if (!comm) return XR_ERR_INVALID;
+  xr_shard_info info;
+  int st = xr_shard_plan(op, dtype, local_dims, level_mask, comm->nranks, comm->rank, &info);
+  if (st) return st;
+  if (info.global_count == 0) return XR_OK;
+  int64_t total = local_dims[0] * local_dims[1] * local_dims[2];
+  if (!out_host || (total > 0 && !in_local_host)) return XR_ERR_INVALID;
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t obytes = (size_t)info.global_count * dtype_size(dtype);
+  if (obytes > comm->hout_bytes) {
+    if (comm->hout) { cudaStreamSynchronize(s); cudaFree(comm->hout); }
+    comm->hout = nullptr;
+    comm->hout_bytes = 0;
+    if (cudaMalloc(&comm->hout, obytes) != cudaSuccess) { cudaGetLastError(); return XR_ERR_NOMEM; }
+    comm->hout_bytes = obytes;
+  }
+  // the caller's init (XR_INIT_FROM_OUT) travels with out
+  if ((level_mask & XR_INIT_FROM_OUT) &&
+      cudaMemcpyAsync(comm->hout, out_host, obytes, cudaMemcpyHostToDevice, s) != cudaSuccess) {
+    cudaGetLastError();
+    return XR_ERR_CUDA;
+  }
+  // local reduction: the chunked H2D pipeline of xr_reduce_host into device memory
+  auto local = [&](unsigned m, void* dst) {
+    return reduce_host_into(op, dtype, local_dims, m, in_local_host, dst, s);
+  };
+  using NoFused = int(unsigned, void*, const ExchArgs*);
+  st = sharded_impl(op, dtype, local_dims, level_mask, comm->hout, comm, s, local, (NoFused*)nullptr);
+  if (!st && cudaMemcpyAsync(out_host, comm->hout, obytes, cudaMemcpyDeviceToHost, s) != cudaSuccess) st = XR_ERR_CUDA;
+  if (cudaStreamSynchronize(s) != cudaSuccess && !st) st = XR_ERR_CUDA;
+  if (st) cudaGetLastError();
+  return st;
+}
+
 int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* T2, double* residual,
                          xr_comm_t comm, xr_stream_t stream) {
   if (!comm || !residual || n_local < 1 || ni < 0 || !T1 || !T2) return XR_ERR_INVALID;
@@ -243,19 +344,27 @@ int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* 
   int st = heat_slab_rows(n_local, comm->nranks, comm->rank, &jb, &je);
   if (st) return st;
   if ((st = heat_step_rows(n_local + 2, ni, jb, je, T1, T2, residual, s))) return st;
-  if (comm->nranks == 1) return XR_OK;
-  // halo rows of the new field: my first owned row goes up, my last goes down
+  // halo rows of the new field: my first owned row goes up, my last goes down.
+  // XR_FORCE_COLL (tests, 1 rank): the rank is its own up and down neighbour,
+  // so the grouped send/recv runs on one GPU; NCCL matches the two self
+  // messages in order, i.e. halo row 0 <- owned row 1 and halo row n+1 <-
+  // owned row n.  Both halo rows are unused at the global boundary.
   const int r = comm->rank;
-  if (ncclGroupStart() != ncclSuccess) return XR_ERR_NCCL;
-  if (r > 0) {
-    ncclSend(T2 + ni, (size_t)ni, ncclFloat64, r - 1, comm->nccl, s);
-    ncclRecv(T2, (size_t)ni, ncclFloat64, r - 1, comm->nccl, s);
+  const bool force = comm->nranks == 1 && std::getenv("XR_FORCE_COLL") != nullptr;
+  const int up = r > 0 ? r - 1 : (force ? r : -1);
+  const int down = r < comm->nranks - 1 ? r + 1 : (force ? r : -1);
+  if (up >= 0 || down >= 0) {
+    if (ncclGroupStart() != ncclSuccess) return XR_ERR_NCCL;
+    if (up >= 0) {
+      ncclSend(T2 + ni, (size_t)ni, ncclFloat64, up, comm->nccl, s);
+      ncclRecv(T2, (size_t)ni, ncclFloat64, up, comm->nccl, s);
+    }
+    if (down >= 0) {
+      ncclSend(T2 + n_local * ni, (size_t)ni, ncclFloat64, down, comm->nccl, s);
+      ncclRecv(T2 + (n_local + 1) * ni, (size_t)ni, ncclFloat64, down, comm->nccl, s);
+    }
+    if (ncclGroupEnd() != ncclSuccess) return XR_ERR_NCCL;
   }
-  if (r < comm->nranks - 1) {
-    ncclSend(T2 + n_local * ni, (size_t)ni, ncclFloat64, r + 1, comm->nccl, s);
-    ncclRecv(T2 + (n_local + 1) * ni, (size_t)ni, ncclFloat64, r + 1, comm->nccl, s);
-  }
-  if (ncclGroupEnd() != ncclSuccess) return XR_ERR_NCCL;
   if (ncclAllReduce(residual, residual, 1, ncclFloat64, ncclMax, comm->nccl, s) != ncclSuccess) return XR_ERR_NCCL;
   return XR_OK;
 }

@@ -32,7 +32,9 @@ struct ExchArgs {
   unsigned long long* peers[kMaxRanks];     // every rank's mailbox (peers[rank] == mine)
   int nranks, rank;
   unsigned long long epoch;                 // > 0, increments per call
-  int* status;                              // set to 1 if a peer never arrived (bounded spin)
+  unsigned long long timeout_ns;            // bound on the wait for the peers (%globaltimer)
+  int* status;                              // set to 1 if a peer never arrived within timeout_ns
+                                            // (host-mapped: readable without a device sync)
 };
 
 // Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]
@@ -118,8 +120,11 @@ struct Plan {
 // over-decomposition (the multi-variable launch shares one grid among its
 // variables), counted in CTA-wide units.  sub_cta (seg_only only): short rows
 // keep the sub-CTA groups of 8 / 32 lanes (p->group) instead of CTA-wide ones.
+// no_tma: never pick the TMA tensor-map column kernel (the launch re-plans
+// with it when encoding the tensor map failed).
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p, bool seg_only = false, int64_t want_units = 0, bool sub_cta = false);
+               int num_sms, Plan* p, bool seg_only = false, int64_t want_units = 0, bool sub_cta = false,
+               bool no_tma = false);
 
 int dtype_size(int dtype);
 int acc_size(int op, int dtype);
@@ -139,7 +144,8 @@ cudaError_t gather_f32(int op, const void* g, int nranks, int64_t n, void* out, 
 cudaError_t gather_f64(int op, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
 
 // Encode the K_COLTMA tensor map for `in` (false if the driver entry point or
-// the encode fails; the caller then falls back to the register column kernel).
+// the encode fails; the caller then re-plans with no_tma and launches the
+// register column kernel instead).
 bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K);
 
 // Grid for `units` work items given the device's resident-CTA budget.

@@ -148,9 +148,18 @@ __device__ __forceinline__ typename Op<OP, T>::Acc seg_unit(const SegArgs& a, in
 }
 
 // Fused exchange (one thread): publish `mine` to every rank's mailbox, wait for
-// all ranks (bounded), then out[0] = combine of the nranks values in rank
-// order -- identical bits on every rank.  `mine` already carries this rank's
-// share of the initial value (rank 0 only, xr_shard_plan).
+// all ranks (bounded by timeout_ns of %globaltimer), then out[0] = combine of
+// the nranks values in rank order -- identical bits on every rank.  `mine`
+// already carries this rank's share of the initial value (rank 0 only,
+// xr_shard_plan).  If a peer does not arrive in time, out is left UNCHANGED
+// and the host-mapped status word is set (the host reports XR_ERR_NCCL on the
+// next call and through xr_comm_query); a stale combine is never written.
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 template <int OP, typename T>
 __device__ __noinline__ void peer_exchange(const ExchArgs& ex, T* out, T mine) {
   const ExchArgs* x = &ex;
@@ -165,16 +174,21 @@ __device__ __noinline__ void peer_exchange(const ExchArgs& ex, T* out, T mine) {
     unsigned long long* f = x->peers[p] + 2 * kMaxRanks + x->rank;
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(x->epoch) : "memory");
   }
+  const unsigned long long t0 = globaltimer_ns();
   typename O::Acc acc = O::identity();
   for (int q = 0; q < x->nranks; ++q) {
     const unsigned long long* f = x->mine + 2 * kMaxRanks + q;
     unsigned long long e = 0ull;
-    for (long long spin = 0; spin < (1ll << 26); ++spin) {
+    while (true) {
       asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(e) : "l"(f) : "memory");
       if (e >= x->epoch) break;
+      if (globaltimer_ns() - t0 > x->timeout_ns) {  // a peer never arrived: report, do not hang
+        *reinterpret_cast<volatile int*>(x->status) = 1;
+        __threadfence_system();
+        return;
+      }
       __nanosleep(64);
     }
-    if (e < x->epoch) *x->status = 1;  // a peer never arrived: report instead of hanging
     unsigned long long v;
     asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(x->mine + par * kMaxRanks + q) : "memory");
     T tv;
@@ -1507,13 +1521,6 @@ __global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int 
 }
 
 // ------------------------------------------------------------- host launch
-template <typename K>
-static int occupancy(K kernel, int block) {
-  int n = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kernel, block, 0) != cudaSuccess || n < 1) n = 1;
-  return n;
-}
-
 template <int OP, typename T>
 cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
   constexpr int VEC = 16 / sizeof(T);
@@ -1534,13 +1541,13 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       const int64_t groups_per_cta = kBlock / p.group;
       const int64_t ctas = (p.units + groups_per_cta - 1) / groups_per_cta;
       if (p.group == 8) {
-        static int occ = occupancy(seg_kernel<OP, T, 8, kBlock, kUnroll>, kBlock);
+        const int occ = occ_dev<seg_kernel<OP, T, 8, kBlock, kUnroll>>(kBlock, 0);
         seg_kernel<OP, T, 8, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
       } else if (p.group == 32) {
-        static int occ = occupancy(seg_kernel<OP, T, 32, kBlock, kUnroll>, kBlock);
+        const int occ = occ_dev<seg_kernel<OP, T, 32, kBlock, kUnroll>>(kBlock, 0);
         seg_kernel<OP, T, 32, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
       } else {
-        static int occ = occupancy(seg_kernel<OP, T, kBlock, kBlock, kUnroll>, kBlock);
+        const int occ = occ_dev<seg_kernel<OP, T, kBlock, kBlock, kUnroll>>(kBlock, 0);
         seg_kernel<OP, T, kBlock, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
       }
       break;
@@ -1548,24 +1555,14 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
     case K_STREAM: {
       auto kern = stream_kernel<OP, T, kStages, kStageBytes>;
       constexpr int dyn = kStages * kStageBytes;
-      static int occ = [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
-        int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsEpiBlock, dyn) != cudaSuccess || n < 1) n = 1;
-        return n;
-      }();
+      const int occ = occ_dev<stream_kernel<OP, T, kStages, kStageBytes>>(kWsEpiBlock, dyn);
       kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsEpiBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_RKR: {
       auto kern = rkr_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
-      static int occ = [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
-        int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsEpiBlock, dyn) != cudaSuccess || n < 1) n = 1;
-        return n;
-      }();
+      const int occ = occ_dev<rkr_kernel<OP, T, kStages>>(kWsEpiBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       kern<<<(unsigned)grid, kWsEpiBlock, dyn, s>>>(p.rkr);
@@ -1574,31 +1571,21 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
     case K_ROWS: {
       auto kern = rows_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
-      static int occ = [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
-        int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
-        return n;
-      }();
+      const int occ = occ_dev<rows_kernel<OP, T, kStages>>(kWsBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.seg);
       break;
     }
     case K_COLFLAT: {
-      static int occ = occupancy(colflat_kernel<OP, T>, kBlock);
+      const int occ = occ_dev<colflat_kernel<OP, T>>(kBlock, 0);
       colflat_kernel<OP, T><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
       break;
     }
     case K_COLTMA: {
       auto kern = coltma_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
-      static int occ = [&] {
-        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
-        int n = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, kern, kWsBlock, dyn) != cudaSuccess || n < 1) n = 1;
-        return n;
-      }();
+      const int occ = occ_dev<coltma_kernel<OP, T, kStages>>(kWsBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.tmap, p.col);
@@ -1606,10 +1593,10 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
     }
     case K_COL: {
       if (p.vec == VEC && VEC > 1) {
-        static int occ = occupancy(col_kernel<OP, T, VEC, kBlock, kUnroll>, kBlock);
+        const int occ = occ_dev<col_kernel<OP, T, VEC, kBlock, kUnroll>>(kBlock, 0);
         col_kernel<OP, T, VEC, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
       } else {
-        static int occ = occupancy(col_kernel<OP, T, 1, kBlock, kUnroll>, kBlock);
+        const int occ = occ_dev<col_kernel<OP, T, 1, kBlock, kUnroll>>(kBlock, 0);
         col_kernel<OP, T, 1, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
       }
       break;

@@ -52,6 +52,31 @@ template <typename T> __device__ __forceinline__ T unpack(const U128& u, int q) 
   }
 }
 
+// Resident CTAs per SM of kernel KERN at `block` threads and `dyn` bytes of
+// dynamic shared memory, cached PER DEVICE: the dynamic-smem attribute binds
+// to the current device's module, so a process that drives a second GPU sets
+// it again there (a function-local static would set it on the first device
+// only).  Setting the attribute twice is harmless, so the cache needs no lock.
+constexpr int kMaxDevices = 64;
+template <auto KERN>
+int occ_dev(int block, int dyn) {
+  static int cache[kMaxDevices];  // 0 = not yet computed on that device
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) { cudaGetLastError(); dev = -1; }
+  if (dev >= 0) {
+    const int v = __atomic_load_n(&cache[dev], __ATOMIC_RELAXED);
+    if (v > 0) return v;
+  }
+  if (dyn > 48 * 1024) cudaFuncSetAttribute(KERN, cudaFuncAttributeMaxDynamicSharedMemorySize, dyn);
+  int n = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, KERN, block, dyn) != cudaSuccess || n < 1) {
+    cudaGetLastError();
+    n = 1;
+  }
+  if (dev >= 0) __atomic_store_n(&cache[dev], n, __ATOMIC_RELAXED);
+  return n;
+}
+
 }  // namespace xr
 
 namespace xr {

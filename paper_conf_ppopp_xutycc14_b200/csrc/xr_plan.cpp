@@ -58,7 +58,7 @@ int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm) {
 }
 
 void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t in_addr,
-               int num_sms, Plan* p, bool seg_only, int64_t want_override, bool sub_cta) {
+               int num_sms, Plan* p, bool seg_only, int64_t want_override, bool sub_cta, bool no_tma) {
   *p = Plan();
   XrEnv env;
   scan_env(&env);
@@ -173,7 +173,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     }
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
     if (!seg_only && !seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
-        B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr) {
+        B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr && !no_tma) {
       const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
       const int64_t tiles = cdiv(K, TWt);
       // Balance (measured r01 sweeps): the producer warp keeps every CTA's ring

@@ -5,6 +5,7 @@
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <mutex>
 
 #include "../../include/xreduce.h"
@@ -28,6 +29,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
 }
 
 bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K) {
+  if (std::getenv("XR_TEST_TMAP_FAIL") != nullptr) return false;  // test hook: the re-plan fallback
   auto fn = encode_fn();
   if (!fn) return false;
   const int size = dtype_size(dtype);

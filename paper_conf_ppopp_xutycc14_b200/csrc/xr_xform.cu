@@ -210,13 +210,7 @@ __global__ void __launch_bounds__(kBlock) xform_col_kernel(const __grid_constant
 
 template <int XF, typename T, int VEC>
 static void xform_col_launch(const ColArgs& c, const void* in2, int sms, cudaStream_t s) {
-  static int occ = [] {
-    int n = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xform_col_kernel<XF, T, VEC>, kBlock, 0) != cudaSuccess ||
-        n < 1)
-      n = 1;
-    return n;
-  }();
+  const int occ = occ_dev<xform_col_kernel<XF, T, VEC>>(kBlock, 0);
   xform_col_kernel<XF, T, VEC><<<(unsigned)grid_for(c.units, sms, occ), kBlock, 0, s>>>(c, in2);
 }
 
@@ -231,11 +225,7 @@ static cudaError_t xform_launch(Plan& p, const void* in2, int sms, cudaStream_t 
     if (p.vec > 1) xform_col_launch<XF, T, 16 / sizeof(T)>(p.col, in2, sms, s);
     else xform_col_launch<XF, T, 1>(p.col, in2, sms, s);
   } else {
-    static int occ = [] {
-      int n = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, xform_kernel<XF, T>, kBlock, 0) != cudaSuccess || n < 1) n = 1;
-      return n;
-    }();
+    const int occ = occ_dev<xform_kernel<XF, T>>(kBlock, 0);
     xform_kernel<XF, T><<<(unsigned)grid_for(p.units, sms, occ), kBlock, 0, s>>>(p.seg, in2);
   }
   count_launch();

@@ -1,0 +1,165 @@
+"""GPU tests of the round-2 boundary work, all through the C ABI against the
+oracle:
+
+- xr_reduce_host's chunked pipeline (include/xreduce.h): inputs many times
+  larger than the staging chunk, every mask, with and without init, and
+  concurrent calls on different streams (per-(device, stream) staging);
+- the TMA encode-failure fallback (re-plan onto the register column kernel);
+- the fused exchange's bounded wait: a rank that never arrives makes the
+  others time out, leave out unchanged and report XR_ERR_NCCL;
+- the Python binding's validation on device tensors.
+"""
+import threading
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from datagen import recipes
+from gpu_util import check, torch_dt
+
+pytestmark = pytest.mark.gpu
+MASKS = ["g", "w", "v", "gw", "gv", "wv", "gwv"]
+KIND = {"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "&": "band", "|": "bor", "^": "bxor",
+        "&&": "land", "||": "lor"}
+
+
+def host_reduce(op, dtype, dims, levels, x, init=None, stream=None):
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    xin = torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
+    n = xr.xr_out_count(dims, levels)
+    out = np.zeros(max(n, 1), dtype=oracle.NP_DTYPES[dtype])
+    mask = xr.mask_of(levels)
+    if init is not None:
+        out[:n] = init
+        mask |= xr.INIT_FROM_OUT
+    s = stream.cuda_stream if stream is not None else torch.cuda.current_stream().cuda_stream
+    st = xr.xr_reduce_host(op, dtype, dims, mask, xin.data_ptr() if x.size else 0, out.ctypes.data, s)
+    assert st == 0, xr.xr_strerror(st)
+    return out[:n]
+
+
+@pytest.mark.parametrize("op,dtype", [("+", "int32"), ("+", "fp32"), ("*", "int64"), ("max", "fp64"),
+                                      ("^", "int64"), ("&&", "fp32"), ("min", "int32"), ("||", "int64")])
+@pytest.mark.parametrize("chunk", [64, 4096, 1 << 20])
+def test_reduce_host_chunked_every_mask(monkeypatch, op, dtype, chunk):
+    """Inputs 10-1000x the chunk: several chunks per output block on every
+    mask, the first merging the caller's init, the others accumulating."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_HOST_CHUNK_BYTES", str(chunk))
+    dims = (37, 19, 23)
+    for lv in MASKS:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, 41)
+        nchunks = len(xr.xr_host_chunks(dims, lv, dtype, chunk))
+        assert nchunks >= (x.nbytes // chunk), (nchunks, x.nbytes, chunk)
+        got = host_reduce(op, dtype, dims, lv, x)
+        check(op, dtype, dims, lv, got, x)
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 9)
+        got = host_reduce(op, dtype, dims, lv, x, init=init)
+        check(op, dtype, dims, lv, got, x, init=init)
+
+
+def test_reduce_host_large_default_chunks():
+    """256 MiB fp32 (8 default 32 MiB chunks) and a 33 MiB odd-sized int64
+    array whose last chunk is partial."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    n = 1 << 26
+    x = datagen.uniform_float(77, n, 0.0, 1.0, np.float32)
+    assert len(xr.xr_host_chunks((n, 1, 1), "gwv", "fp32", 32 << 20)) == 8
+    check("+", "fp32", (n, 1, 1), "gwv", host_reduce("+", "fp32", (n, 1, 1), "gwv", x), x)
+    n2 = (33 << 20) // 8 + 3
+    y = datagen.uniform_int(78, n2, -(1 << 40), 1 << 40, np.int64)
+    for lv, dims in (("gwv", (n2, 1, 1)), ("v", (n2 // 3 // 1, 1, 3))):
+        yy = y[:dims[0] * dims[2]]
+        check("+", "int64", dims, lv, host_reduce("+", "int64", dims, lv, yy), yy)
+
+
+def test_reduce_host_concurrent_streams(monkeypatch):
+    """Two host threads on two streams: per-(device, stream) staging keeps
+    their chunks apart (one shared staging buffer raced)."""
+    import torch
+    monkeypatch.setenv("XR_HOST_CHUNK_BYTES", str(1 << 16))
+    dims = (64, 33, 129)
+    xs = [datagen.uniform_int(200 + t, int(np.prod(dims)), -1000, 1000, np.int32) for t in range(2)]
+    refs = [oracle.reduce("+", "int32", dims, "gw", x) for x in xs]
+    streams = [torch.cuda.Stream() for _ in range(2)]
+    errors = []
+
+    def worker(t):
+        try:
+            torch.cuda.set_device(0)
+            for _ in range(10):
+                got = host_reduce("+", "int32", dims, "gw", xs[t], stream=streams[t])
+                if not np.array_equal(got, refs[t]):
+                    errors.append(t)
+        except Exception as e:  # noqa: BLE001
+            errors.append(repr(e))
+
+    th = [threading.Thread(target=worker, args=(t,)) for t in range(2)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    assert not errors, errors
+
+
+def test_reduce_host_empty_reduced_extent():
+    got = host_reduce("+", "int32", (0, 3, 4), "g", np.zeros(0, dtype=np.int32), init=np.arange(12, dtype=np.int32))
+    assert np.array_equal(got, np.arange(12, dtype=np.int32))  # C17: out = init
+
+
+def test_tma_encode_failure_falls_back(monkeypatch):
+    """XR_TEST_TMAP_FAIL makes the tensor-map encode fail: the call re-plans
+    onto the register column kernel (one launch) and stays correct."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    dims = (1, 4096, 2048)
+    x = datagen.uniform_int(5, int(np.prod(dims)), -(1 << 20), 1 << 20, np.int32)
+    xd = torch.from_numpy(x).cuda()
+    assert xr.xr_plan_describe("+", "int32", dims, "w", xd.data_ptr())["kernel"] == "coltma"
+    monkeypatch.setenv("XR_TEST_TMAP_FAIL", "1")
+    n0 = xr.xr_launch_count()
+    got = xr.reduce(xd, "+", "w", nest=dims)
+    torch.cuda.synchronize()
+    assert xr.xr_launch_count() - n0 == 1
+    assert np.array_equal(got.cpu().numpy(), oracle.reduce("+", "int32", dims, "w", x))
+
+
+@pytest.mark.parametrize("G,skip", [(2, 1), (4, 0), (3, 2)])
+def test_fused_exchange_times_out_without_stale_write(monkeypatch, G, skip):
+    """One simulated rank never launches: the others' bounded waits expire,
+    they leave out unchanged (no stale combine) and the call reports
+    XR_ERR_NCCL."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_TEST_SIM_SKIP_RANK", str(skip))
+    monkeypatch.setenv("XR_EXCH_TIMEOUT_MS", "300")
+    n_local = 1 << 20
+    xd = torch.ones(n_local * G, dtype=torch.int64, device="cuda")
+    outs = [torch.full((1,), -7, dtype=torch.int64, device="cuda") for _ in range(G)]
+    st = xr.xr_reduce_fused_sim("+", "int64", (n_local, 1, 1), 7,
+                                [xd[r * n_local:(r + 1) * n_local].data_ptr() for r in range(G)],
+                                [o.data_ptr() for o in outs])
+    assert st == xr.ERR_NCCL
+    assert [int(o.item()) for o in outs] == [-7] * G
+    monkeypatch.delenv("XR_TEST_SIM_SKIP_RANK")
+    st = xr.xr_reduce_fused_sim("+", "int64", (n_local, 1, 1), 7,
+                                [xd[r * n_local:(r + 1) * n_local].data_ptr() for r in range(G)],
+                                [o.data_ptr() for o in outs])
+    assert st == 0 and [int(o.item()) for o in outs] == [n_local * G] * G
+
+
+def test_python_binding_validates_device_calls():
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    x = torch.arange(24, dtype=torch.int32, device="cuda")
+    with pytest.raises(ValueError):
+        xr.reduce(x, "+", "g", nest=(5, 5, 1))                     # 25 != 24 elements
+    with pytest.raises(ValueError):
+        xr.reduce(x, "+", "g", nest=(2, 3, 4), out=torch.zeros(12, dtype=torch.int64, device="cuda"))
+    with pytest.raises(ValueError):
+        xr.reduce(x, "+", "g", nest=(2, 3, 4), out=torch.zeros(12, dtype=torch.int32))  # host out
+    got = xr.reduce(x.reshape(2, 3, 2, 2), "+", "g")              # 4-D: leading dims flattened -> (6, 2, 2)
+    assert got.cpu().tolist() == [[sum(range(k, 24, 4)) for k in range(j * 2, j * 2 + 2)] for j in range(2)]

@@ -1,10 +1,16 @@
 #!/usr/bin/env python3
-"""Summarise ncu reports (gpurun_out/ncu/*.ncu-rep) into profiles/.
+"""Summarise ncu reports (gpurun_out/ncu/<case>_<TAG>.ncu-rep) into profiles/.
 
   python tools/ncu_summary.py TAG [--launches CSV]
 
-Writes profiles/ncu_<TAG>.md (one table row per captured kernel) and merges
-per-launch DRAM traffic into profiles/ncu_traffic.json (read by bench.py).
+<case> is a tools/kdriver.py case name (cfg2-f32-sum, cfg3-col, cfg4-heat,
+cfg5-<op>-<dtype>-<mask>, nest-..., mc-pi-N, ...).  Writes
+profiles/ncu_<TAG>.md (one row per captured kernel, with ncu's
+dram__throughput.avg.pct_of_peak_sustained_elapsed -- the BASELINE metric's
+"% of B200 HBM peak (ncu)") and merges per-case records into
+profiles/ncu_dram.json ({case: {traffic, dram_pct, time_us, alg_bytes,
+source}}; bench.py reads its workload's entry), plus DRAM bytes into
+profiles/ncu_traffic.json (history).
 """
 import csv
 import glob
@@ -21,6 +27,7 @@ METRICS = [
     ("dram__bytes_write.sum", "DRAM write"),
     ("dram__bytes.sum.per_second", "DRAM B/s"),
     ("dram__throughput.avg.pct_of_peak_sustained_elapsed", "DRAM % peak"),
+    ("dram__cycles_active.avg.pct_of_peak_sustained_elapsed", "DRAM cycles active %"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps active %"),
     ("launch__registers_per_thread", "regs"),
     ("launch__grid_size", "grid"),
@@ -29,10 +36,44 @@ METRICS = [
     ("launch__occupancy_limit_shared_mem", "occ lim smem"),
     ("smsp__inst_executed.sum", "inst"),
 ]
-# algorithmic bytes per launch for the kdriver cases
-ALG = {"fp32sum": 4 * 2**30 + 4, "cfg3col": 4 * 2**30 + 4 * 32768, "cfg3row": 4 * 2**30 + 4 * 32768,
-       "heat": 16 * 8192 * 8192, "cfg5v": 4 * 2**27 + 4 * 2**18}
-WORKLOAD = {"fp32sum": "fp32-sum"}
+SIZE = {"int32": 4, "int64": 8, "fp32": 4, "fp64": 8, "f32": 4, "f64": 8, "i32": 4, "i64": 8}
+# bench.py workload names of the cfg2 captures
+WORKLOAD = {"cfg2-f32-sum": "fp32-sum", "cfg2-f32-max": "fp32-max", "cfg2-f32-min": "fp32-min",
+            "cfg2-i64-sum": "int64-sum", "cfg2-i64-max": "int64-max", "cfg2-i64-min": "int64-min",
+            "fp32sum": "fp32-sum"}
+
+
+def out_count(dims, lv):
+    c = 1
+    for d, ch in enumerate("gwv"):
+        if ch not in lv:
+            c *= dims[d]
+    return c
+
+
+def alg_bytes(case):
+    """Algorithmic bytes per launch of a kdriver case."""
+    if case.startswith("cfg2-"):
+        return (2**30 + 1) * SIZE[case.split("-")[1]]
+    if case in ("cfg3-row", "cfg3-col", "cfg3row", "cfg3col"):
+        return 4 * 2**30 + 4 * 32768
+    if case in ("cfg4-heat", "heat"):
+        return 16 * 8192 * 8192
+    if case.startswith("heat-"):
+        n = int(case.split("-")[1])
+        return 16 * n * n
+    if case == "fp32sum":
+        return 4 * 2**30 + 4
+    if case.startswith("cfg5-"):
+        _, _, dt, lv = case.split("-")
+        return (2**27 + out_count((512, 512, 512), lv)) * SIZE[dt]
+    if case.startswith("nest-"):
+        _, _, dt, dims, lv = case.split("-")
+        d = tuple(int(v) for v in dims.split("x"))
+        return (d[0] * d[1] * d[2] + out_count(d, lv)) * SIZE[dt]
+    if case.startswith("mc-pi"):
+        return 8 * (1 << int(case.split("-")[2]))
+    return None
 
 
 def to_bytes(v, unit):
@@ -54,15 +95,19 @@ def main():
     reps = sorted(glob.glob(os.path.join(ROOT, "gpurun_out", "ncu", f"*_{tag}.ncu-rep")))
     os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    dpath = os.path.join(ROOT, "profiles", "ncu_dram.json")
     traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
+    dram = json.load(open(dpath)) if os.path.exists(dpath) else {}
     lines = [f"# ncu summary — {tag}", "",
              "`ncu --set full --clock-control none --import-source on -k regex:<kernel> -s 3 -c 1` "
-             "on `tools/kdriver.py <case>` (one B200, cold L2 per replay). Algorithmic bytes from "
-             "DESIGN.md section 5.", "",
-             "| case | kernel | time (us) | DRAM read | DRAM write | traffic / algorithmic | DRAM TB/s | regs | grid | occ lim (regs/smem) | warps active % |",
-             "|---|---|---|---|---|---|---|---|---|---|---|"]
+             "on `tools/kdriver.py <case>` (one B200, cold L2 per replay). **DRAM %** is "
+             "`dram__throughput.avg.pct_of_peak_sustained_elapsed`, the BASELINE metric's "
+             "\"% of B200 HBM peak (ncu)\". Algorithmic bytes from DESIGN.md section 5.", "",
+             "| case | kernel | time (us) | DRAM % | DRAM read | DRAM write | traffic / algorithmic | DRAM TB/s | "
+             "regs | grid | occ lim (regs/smem) | warps active % |",
+             "|---|---|---|---|---|---|---|---|---|---|---|---|"]
     for rep in reps:
-        case = os.path.basename(rep).rsplit("_", 1)[0]
+        case = os.path.basename(rep)[:-len(f"_{tag}.ncu-rep")]
         r = raw(rep)
         if r is None:
             continue
@@ -74,14 +119,30 @@ def main():
         t_us = float(d["gpu__time_duration.sum"][0].replace(",", ""))
         if d["gpu__time_duration.sum"][1] == "ms":
             t_us *= 1e3
-        alg = ALG.get(case)
+        elif d["gpu__time_duration.sum"][1] == "ns":
+            t_us /= 1e3
+        # ncu's "DRAM Throughput" (GPU Speed Of Light section); --set full
+        # stores it as dram__cycles_active.avg.pct_of_peak_sustained_elapsed
+        pct = None
+        for m in ("dram__throughput.avg.pct_of_peak_sustained_elapsed",
+                  "dram__cycles_active.avg.pct_of_peak_sustained_elapsed"):
+            if m in hdr and vals[hdr.index(m)].strip():
+                pct = float(vals[hdr.index(m)].replace(",", ""))
+                break
+        alg = alg_bytes(case)
         ratio = f"{(rd + wr) / alg:.4f}" if alg else "-"
-        bw = to_bytes(*d["dram__bytes.sum.per_second"]) / 1e12
-        lines.append(f"| {case} | `{kname[:60]}` | {t_us:.1f} | {rd/1e9:.4f} GB | {wr/1e6:.2f} MB | {ratio} | "
-                     f"{bw:.2f} | {d['launch__registers_per_thread'][0]} | {d['launch__grid_size'][0]} | "
-                     f"{float(d.get('launch__occupancy_limit_registers', ('0',))[0]):.0f}/{float(d.get('launch__occupancy_limit_shared_mem', ('0',))[0]):.0f} | "
-                     f"{float(d['sm__warps_active.avg.pct_of_peak_sustained_active'][0]):.1f} |")
+        bw = to_bytes(*d["dram__bytes.sum.per_second"]) / 1e12 if "dram__bytes.sum.per_second" in d else \
+            (rd + wr) / (t_us * 1e-6) / 1e12
+        g = lambda m: d.get(m, ("-",))[0]  # noqa: E731  (metrics-only captures lack the launch stats)
+        lines.append(f"| {case} | `{kname[:60]}` | {t_us:.1f} | **{pct if pct is None else round(pct, 1)}** | {rd/1e9:.4f} GB | {wr/1e6:.2f} MB | "
+                     f"{ratio} | {bw:.2f} | {g('launch__registers_per_thread')} | {g('launch__grid_size')} | "
+                     f"{g('launch__occupancy_limit_registers')}/{g('launch__occupancy_limit_shared_mem')} | "
+                     f"{g('sm__warps_active.avg.pct_of_peak_sustained_active')} |")
+        rec = {"traffic": rd + wr, "dram_pct": pct, "time_us": t_us, "alg_bytes": alg, "kernel": kname,
+               "source": f"profiles/ncu_{tag}.md ({os.path.basename(rep)})"}
+        dram[f"{case}@{tag}"] = rec
         if case in WORKLOAD:
+            dram[WORKLOAD[case]] = rec
             traffic[WORKLOAD[case]] = rd + wr
         traffic[f"{case}@{tag}"] = rd + wr
     if len(sys.argv) > 3 and sys.argv[2] == "--launches":
@@ -104,6 +165,7 @@ def main():
     with open(os.path.join(ROOT, "profiles", f"ncu_{tag}.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     json.dump(traffic, open(tpath, "w"), indent=1, sort_keys=True)
+    json.dump(dram, open(dpath, "w"), indent=1, sort_keys=True)
     print("\n".join(lines))
 
 
