@@ -270,12 +270,16 @@ def run_reference(args):
 
 
 # --------------------------------------------------------------------- GPU arm
-def timed_loop(step, steps, stream, world):
+def timed_loop(step, steps, stream, world, per_step=True):
     """K steps bracketed by barrier + synchronize; returns (max-over-ranks ms
-    of the whole loop, per-step event ms on this rank)."""
+    of the whole loop, per-step event ms on this rank).  per_step=False keeps
+    event records out of the stream between steps, so back-to-back launches
+    can overlap one launch's drain with the next one's start (programmatic
+    dependent launch); the per-step list is then empty."""
     import torch
     import torch.distributed as dist
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(steps if per_step else 0)]
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
     if world > 1:
@@ -283,9 +287,11 @@ def timed_loop(step, steps, stream, world):
     torch.cuda.synchronize()
     t0.record(stream)
     for i in range(steps):
-        ev[i][0].record(stream)
+        if per_step:
+            ev[i][0].record(stream)
         step()
-        ev[i][1].record(stream)
+        if per_step:
+            ev[i][1].record(stream)
     t1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -398,19 +404,19 @@ def run_gpu(args):
     clocks.start()
     time.sleep(0.3)  # let the sampler attach
     launches0 = xr.xr_launch_count()
-    total_ms, per = timed_loop(step, args.steps, stream, world)
+    total_ms, _ = timed_loop(step, args.steps, stream, world, per_step=False)
     launches = xr.xr_launch_count() - launches0
     ck = clocks.stop()
     ms_step = total_ms / args.steps
     value = total * args.steps / (total_ms / 1e3)
 
-    # kernel-only duration on this rank: at N=1 the step IS the one reduction
-    # kernel; at N>1 the local kernel is timed alone as well (no exchange)
+    # the dominant kernel's average launch duration (roofline.achieved): the
+    # local reduction timed alone, one CUDA-event pair per launch (so launches
+    # do not overlap); at N>1 this is also the kernel-only time without exchange
+    loc_total, per = timed_loop(local_step, args.steps, stream, world)
     kern_ms = statistics.mean(per)
     multi = None
     if use_comm:  # N>1 (or --force-comm at N=1, which exercises the same code)
-        loc_total, loc_per = timed_loop(local_step, args.steps, stream, world)
-        kern_ms = statistics.mean(loc_per)
         # 1-GPU reference time in the same run: rank 0 reduces the whole
         # strong-scaling array (its own slice repeated: timing does not depend
         # on the values) or, weak, its own slice

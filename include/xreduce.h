@@ -270,6 +270,14 @@ int xr_shutdown(void);
 /* Number of kernels this library has launched in this process. */
 int64_t xr_launch_count(void);
 
+/* Profiling only: while buf (DEVICE, 2 + 2*cap_records uint64 words) is set,
+ * the stream kernel appends per-CTA timeline records -- word 0 = records
+ * written (the caller zeroes it), word 1 = cap_records (the caller writes
+ * it), then per record {cta << 40 | event << 32 | unit, %globaltimer ns} with
+ * events 0 CTA start, 1 unit claimed, 2 unit folded, 3 consumers done, 4 last
+ * CTA fold begins, 5 output written.  buf = NULL switches it off. */
+int xr_debug_timeline(void* buf, int64_t cap_records);
+
 /* --------------------------------------------------------- heat (cfg 4) ---- */
 
 /* One fused Jacobi sweep + max-residual reduction of the 2-D heat equation

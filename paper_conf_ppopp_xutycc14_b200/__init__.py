@@ -95,6 +95,7 @@ _SIGS = {
     "xr_reserve": (_c, [_c, _c, _i64p, _u, _vp]),
     "xr_shutdown": (_c, []),
     "xr_launch_count": (ctypes.c_int64, []),
+    "xr_debug_timeline": (_c, [_vp, ctypes.c_int64]),
     "xr_heat_step": (_c, [ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp]),
     "xr_heat_run": (_c, [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, _vp, _vp, _vp, _vp]),
     "xr_shard_plan": (_c, [_c, _c, _i64p, _u, _c, _c, ctypes.POINTER(ShardInfo)]),

@@ -18,6 +18,8 @@ namespace xr {
 
 static std::atomic<int64_t> g_launches{0};
 void count_launch() { g_launches.fetch_add(1, std::memory_order_relaxed); }
+static std::atomic<unsigned long long*> g_timeline{nullptr};
+unsigned long long* debug_timeline() { return g_timeline.load(std::memory_order_relaxed); }
 
 static bool is_fp(int dtype) { return dtype == XR_FP32 || dtype == XR_FP64; }
 
@@ -161,6 +163,7 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   const int ifo = (mask & XR_INIT_FROM_OUT) ? 1 : 0;
   p.seg.in = in; p.seg.out = out; p.seg.partials = w.partials; p.seg.tickets = w.tickets;
   p.seg.init_from_out = ifo;
+  p.seg.tl = debug_timeline();
   p.col.in = in; p.col.out = out; p.col.partials = w.partials; p.col.tickets = w.tickets;
   p.col.init_from_out = ifo;
   p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
@@ -505,6 +508,12 @@ int xr_shutdown(void) {
 }
 
 int64_t xr_launch_count(void) { return g_launches.load(); }
+
+int xr_debug_timeline(void* buf, int64_t cap_records) {
+  if (buf && cap_records < 1) return XR_ERR_INVALID;
+  g_timeline.store(static_cast<unsigned long long*>(buf), std::memory_order_relaxed);
+  return XR_OK;
+}
 
 int xr_reduce_host(int op, int dtype, const int64_t nest_dims[3], unsigned level_mask,
                    const void* in_host, void* out_host, xr_stream_t stream) {

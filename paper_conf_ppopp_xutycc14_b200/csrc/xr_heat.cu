@@ -56,6 +56,8 @@ __device__ __forceinline__ double ld_row(const double* p) { return __ldg(p); }
 // peak in profiles/ r01).
 template <int VEC>
 __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP_MAX, double>;
   constexpr int NW = kBlock / 32;
   constexpr int STRIP = 32 * VEC;
@@ -191,6 +193,8 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   if (warp == 0) {
     // producer warp: row q of the tile into slot q % kHeatSlots once the
     // consumers released the row kHeatSlots earlier
@@ -307,6 +311,8 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
       int64_t q = 0;  // global row counter (slot = q % kHeatSlots)
@@ -474,6 +480,7 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   a.tickets = tickets;
   dim3 grid((unsigned)gx, (unsigned)gy);
   const char* hp = std::getenv("XR_HEAT_ONE_TILE");  // A/B: one tile per CTA
+  cudaError_t le = cudaSuccess;
   if (bulk && hp == nullptr && je > jb) {
     auto occ_of = [](auto kern) {
       int n = 0;
@@ -492,13 +499,13 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
     pa.gy = gy;
     pa.sched = reinterpret_cast<unsigned long long*>(tickets + 2);  // after the residual ticket (8-B aligned)
     const int64_t pgrid = std::min<int64_t>(gx * gy, (int64_t)sms * occ);
-    if (odd) heat_persistent_kernel<true><<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
-    else heat_persistent_kernel<false><<<(unsigned)pgrid, kWsBlock, 0, s>>>(pa);
-  } else if (bulk) heat_bulk_kernel<<<grid, kWsBlock, 0, s>>>(a);
-  else if (v2) heat_kernel<2><<<grid, kBlock, 0, s>>>(a);
-  else heat_kernel<1><<<grid, kBlock, 0, s>>>(a);
+    if (odd) le = launch_pdl(heat_persistent_kernel<true>, dim3((unsigned)pgrid), dim3(kWsBlock), 0, s, pa);
+    else le = launch_pdl(heat_persistent_kernel<false>, dim3((unsigned)pgrid), dim3(kWsBlock), 0, s, pa);
+  } else if (bulk) le = launch_pdl(heat_bulk_kernel, grid, dim3(kWsBlock), 0, s, a);
+  else if (v2) le = launch_pdl(heat_kernel<2>, grid, dim3(kBlock), 0, s, a);
+  else le = launch_pdl(heat_kernel<1>, grid, dim3(kBlock), 0, s, a);
   count_launch();
-  if (cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  if (le != cudaSuccess || cudaPeekAtLastError() != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
   return XR_OK;
 }
 

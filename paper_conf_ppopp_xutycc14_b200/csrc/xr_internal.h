@@ -37,6 +37,20 @@ struct ExchArgs {
                                             // (host-mapped: readable without a device sync)
 };
 
+// Guided unit schedule of the stream kernel's whole-array (R) shape: phase k
+// holds units [u0[k], u0[k+1]) of len[k] elements each, starting at element
+// c0[k] (the last unit of a phase ends at c0[k+1]).  Early phases hand every
+// CTA a long unit (half the remaining work per phase), the last phase short
+// ones, so the CTAs finish within about one short unit of each other while
+// the number of unit partials (and the last CTA's fold) stays small.
+constexpr int kMaxPhases = 12;
+struct Guided {
+  int nph;                       // 0: equal units (Sr x Sc split)
+  int64_t u0[kMaxPhases + 1];
+  int64_t c0[kMaxPhases + 1];
+  int64_t len[kMaxPhases];
+};
+
 // Segmented rows ("seg"): out[o] = (+)_{r<C} (+)_{i<L} in[o*oStride + r*rowStride + i]
 // -- covers R (O=1, C=1), KR (C=1) and RKR (C = outer reduced extent).
 struct SegArgs {
@@ -51,6 +65,8 @@ struct SegArgs {
   int init_from_out;
   int use_exch;          // 1: fused exchange of the O == 1 result (exch below)
   ExchArgs exch;
+  unsigned long long* tl;  // profiling timeline (xr_debug_timeline), null when off
+  Guided gd;               // stream kernel, R shape: guided units (gd.nph > 0)
 };
 
 // Columns ("col"): out[b][c] = (+)_{r<R} in[b][r][c]  -- covers RK (B=1) and KRK.
@@ -152,5 +168,8 @@ bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t
 int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm);
 
 void count_launch();
+
+// The profiling timeline buffer set by xr_debug_timeline (null when off).
+unsigned long long* debug_timeline();
 
 }  // namespace xr

@@ -9,6 +9,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "xr_internal.h"
 #include "xr_ops.cuh"
@@ -154,12 +155,6 @@ __device__ __forceinline__ typename Op<OP, T>::Acc seg_unit(const SegArgs& a, in
 // xr_shard_plan).  If a peer does not arrive in time, out is left UNCHANGED
 // and the host-mapped status word is set (the host reports XR_ERR_NCCL on the
 // next call and through xr_comm_query); a stale combine is never written.
-__device__ __forceinline__ unsigned long long globaltimer_ns() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
-
 template <int OP, typename T>
 __device__ __noinline__ void peer_exchange(const ExchArgs& ex, T* out, T mine) {
   const ExchArgs* x = &ex;
@@ -274,6 +269,8 @@ template <int OP, typename T, int W, int BLOCK, int U>
 #define XR_SEG_MINB 4
 #endif
 __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_constant__ SegArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   __shared__ Acc smem[32];
@@ -399,10 +396,20 @@ __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u)
     g.nbody = (r1 - r0) * a.L;
     return g;
   }
-  const int64_t S = a.Sc;
-  g.o = u / S;
-  const int64_t s = u - g.o * S;
-  const int64_t c0 = split_lo_vec(a.L, S, s, VEC), c1 = split_lo_vec(a.L, S, s + 1, VEC);
+  int64_t c0, c1;
+  if (a.gd.nph > 0) {  // guided units of the whole-array shape (O == 1)
+    int k = 0;
+    while (k + 1 < a.gd.nph && u >= a.gd.u0[k + 1]) ++k;
+    g.o = 0;
+    c0 = a.gd.c0[k] + (u - a.gd.u0[k]) * a.gd.len[k];
+    c1 = min(c0 + a.gd.len[k], a.gd.c0[k + 1]);
+  } else {
+    const int64_t S = a.Sc;
+    g.o = u / S;
+    const int64_t s = u - g.o * S;
+    c0 = split_lo_vec(a.L, S, s, VEC);
+    c1 = split_lo_vec(a.L, S, s + 1, VEC);
+  }
   const T* row = static_cast<const T*>(a.in) + g.o * a.oStride + c0;
   const int64_t n = c1 - c0;
   int64_t head = (int64_t)((16u - ((uint32_t)(uintptr_t)row & 15u)) & 15u) / (int64_t)sizeof(T);
@@ -455,16 +462,20 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
 
   if (warp == 0) {
     // ---------------- producer warp: claims units, publishes their ids and
     // streams their 16-B aligned bodies into the ring NS stages ahead; it never
     // waits for the consumers' epilogues, only for a stage to be released.
     if (lane == 0) {
+      tl_event(a.tl, TL_START, 0);
       int64_t g = 0;
       int seq = 0;
       long long u = claim_first(a.sched);
       while (true) {
+        tl_event(a.tl, TL_UNIT, u);
         const long long nu = claim_next(a.sched);  // next claim, in flight
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < a.units ? u : -1;
@@ -595,6 +606,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
     // only after the barrier of unit n+1, i.e. after warp 0 read unit n's
     v = cons_reduce<OP, T>(v, smem + (seq & 1) * kConsWarps, cw, lane);
     const int64_t o = geo.o;
+    if (ct == 0) tl_event(a.tl, TL_UNIT_DONE, u);
     if (whole) {
       if (ct == 0) partials[u] = v;
     } else if (S == 1) {
@@ -614,6 +626,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
     box_u[slot] = -1;
     mbar_arrive(&bfull[slot]);
   }
+  if (ct == 0) tl_event(a.tl, TL_CONS_END, 0);
   if (whole) {  // a4: one ticket per CTA; the last CTA folds the S unit partials in unit order
     if (ct == 0) {
       const unsigned t = ticket_add(&a.tickets[0]);
@@ -621,6 +634,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
     }
     cons_sync();
     if (s_last) {
+      if (ct == 0) tl_event(a.tl, TL_FOLD, 0);
       __threadfence();
       Acc w = fold_partials_vec<OP, T>(partials, S, ct, kConsThreads);
       w = cons_reduce<OP, T>(w, smem, cw, lane);
@@ -629,6 +643,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
         a.tickets[0] = 0u;
         if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
         else out[0] = r;
+        tl_event(a.tl, TL_END, 0);
       }
     }
   }
@@ -672,6 +687,8 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
 
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
@@ -769,6 +786,8 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
 // paper's 2^20 x 2 x 32 gang case).
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __grid_constant__ ColArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -981,6 +1000,8 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
 
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
@@ -1153,6 +1174,8 @@ template <int OP, typename T, int VEC, int BLOCK, int U>
 #define XR_COL_MINB 1
 #endif
 __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_constant__ ColArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int NW = BLOCK / 32;
@@ -1319,6 +1342,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     fence_mbar_init();
   }
   __syncthreads();
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
 
   if (warp == 0) {
     // ---------------- producer warp
@@ -1494,6 +1519,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
 // ------------------------------------------------------------- elementwise
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   const T* in = static_cast<const T*>(a.in);
   T* out = static_cast<T*>(a.out);
@@ -1503,6 +1530,8 @@ __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
 
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) fill_kernel(EltArgs a) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   T* out = static_cast<T*>(a.out);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (int64_t)gridDim.x * blockDim.x)
@@ -1512,6 +1541,8 @@ __global__ void __launch_bounds__(kBlock) fill_kernel(EltArgs a) {
 // Fixed rank-order combine of gathered partial results (sharded path).
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int nranks, int64_t n, T* out) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using O = Op<OP, T>;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     typename O::Acc v = O::identity();
@@ -1521,6 +1552,7 @@ __global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int 
 }
 
 // ------------------------------------------------------------- host launch
+
 template <int OP, typename T>
 cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
   constexpr int VEC = 16 / sizeof(T);
@@ -1529,12 +1561,12 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       return cudaSuccess;
     case K_FILL: {
       const int64_t grid = grid_for((p.elt.n + kBlock - 1) / kBlock, num_sms, 8);
-      fill_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(p.elt);
+      if (cudaError_t e = launch_pdl(fill_kernel<OP, T>, dim3((unsigned)grid), dim3(kBlock), 0, s, p.elt)) return e;
       break;
     }
     case K_IDENT: {
       const int64_t grid = grid_for((p.elt.n + kBlock - 1) / kBlock, num_sms, 8);
-      ident_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(p.elt);
+      if (cudaError_t e = launch_pdl(ident_kernel<OP, T>, dim3((unsigned)grid), dim3(kBlock), 0, s, p.elt)) return e;
       break;
     }
     case K_SEG: {
@@ -1542,13 +1574,13 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       const int64_t ctas = (p.units + groups_per_cta - 1) / groups_per_cta;
       if (p.group == 8) {
         const int occ = occ_dev<seg_kernel<OP, T, 8, kBlock, kUnroll>>(kBlock, 0);
-        seg_kernel<OP, T, 8, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+        if (cudaError_t e = launch_pdl(seg_kernel<OP, T, 8, kBlock, kUnroll>, dim3((unsigned)grid_for(ctas, num_sms, occ)), dim3(kBlock), 0, s, p.seg)) return e;
       } else if (p.group == 32) {
         const int occ = occ_dev<seg_kernel<OP, T, 32, kBlock, kUnroll>>(kBlock, 0);
-        seg_kernel<OP, T, 32, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+        if (cudaError_t e = launch_pdl(seg_kernel<OP, T, 32, kBlock, kUnroll>, dim3((unsigned)grid_for(ctas, num_sms, occ)), dim3(kBlock), 0, s, p.seg)) return e;
       } else {
         const int occ = occ_dev<seg_kernel<OP, T, kBlock, kBlock, kUnroll>>(kBlock, 0);
-        seg_kernel<OP, T, kBlock, kBlock, kUnroll><<<(unsigned)grid_for(ctas, num_sms, occ), kBlock, 0, s>>>(p.seg);
+        if (cudaError_t e = launch_pdl(seg_kernel<OP, T, kBlock, kBlock, kUnroll>, dim3((unsigned)grid_for(ctas, num_sms, occ)), dim3(kBlock), 0, s, p.seg)) return e;
       }
       break;
     }
@@ -1556,7 +1588,9 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       auto kern = stream_kernel<OP, T, kStages, kStageBytes>;
       constexpr int dyn = kStages * kStageBytes;
       const int occ = occ_dev<stream_kernel<OP, T, kStages, kStageBytes>>(kWsEpiBlock, dyn);
-      kern<<<(unsigned)grid_for(p.units, num_sms, occ), kWsEpiBlock, dyn, s>>>(p.seg);
+      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kWsEpiBlock), dyn, s,
+                                     p.seg))
+        return e;
       break;
     }
     case K_RKR: {
@@ -1565,7 +1599,7 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       const int occ = occ_dev<rkr_kernel<OP, T, kStages>>(kWsEpiBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      kern<<<(unsigned)grid, kWsEpiBlock, dyn, s>>>(p.rkr);
+      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsEpiBlock), dyn, s, p.rkr)) return e;
       break;
     }
     case K_ROWS: {
@@ -1574,12 +1608,12 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       const int occ = occ_dev<rows_kernel<OP, T, kStages>>(kWsBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.seg);
+      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.seg)) return e;
       break;
     }
     case K_COLFLAT: {
       const int occ = occ_dev<colflat_kernel<OP, T>>(kBlock, 0);
-      colflat_kernel<OP, T><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
+      if (cudaError_t e = launch_pdl(colflat_kernel<OP, T>, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kBlock), 0, s, p.col)) return e;
       break;
     }
     case K_COLTMA: {
@@ -1588,16 +1622,16 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       const int occ = occ_dev<coltma_kernel<OP, T, kStages>>(kWsBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      kern<<<(unsigned)grid, kWsBlock, dyn, s>>>(p.tmap, p.col);
+      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.tmap, p.col)) return e;
       break;
     }
     case K_COL: {
       if (p.vec == VEC && VEC > 1) {
         const int occ = occ_dev<col_kernel<OP, T, VEC, kBlock, kUnroll>>(kBlock, 0);
-        col_kernel<OP, T, VEC, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
+        if (cudaError_t e = launch_pdl(col_kernel<OP, T, VEC, kBlock, kUnroll>, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kBlock), 0, s, p.col)) return e;
       } else {
         const int occ = occ_dev<col_kernel<OP, T, 1, kBlock, kUnroll>>(kBlock, 0);
-        col_kernel<OP, T, 1, kBlock, kUnroll><<<(unsigned)grid_for(p.units, num_sms, occ), kBlock, 0, s>>>(p.col);
+        if (cudaError_t e = launch_pdl(col_kernel<OP, T, 1, kBlock, kUnroll>, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kBlock), 0, s, p.col)) return e;
       }
       break;
     }
@@ -1611,8 +1645,9 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
 template <int OP, typename T>
 cudaError_t launch_gather_typed(const void* g, int nranks, int64_t n, void* out, cudaStream_t s) {
   const int64_t grid = std::max<int64_t>(1, std::min<int64_t>((n + kBlock - 1) / kBlock, 148 * 8));
-  gather_combine_kernel<OP, T><<<(unsigned)grid, kBlock, 0, s>>>(static_cast<const T*>(g), nranks, n,
-                                                                  static_cast<T*>(out));
+  if (cudaError_t e = launch_pdl(gather_combine_kernel<OP, T>, dim3((unsigned)grid), dim3(kBlock), 0, s,
+                                 static_cast<const T*>(g), nranks, n, static_cast<T*>(out)))
+    return e;
   count_launch();
   return cudaPeekAtLastError();
 }

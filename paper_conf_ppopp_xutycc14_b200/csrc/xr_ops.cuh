@@ -2,6 +2,7 @@
 // copies, mbarriers, warp specialisation).  The operator traits and the
 // reduction tiers live in the public include/xreduce_device.cuh.
 #pragma once
+#include <cstdlib>
 #include "../../include/xreduce_device.cuh"
 
 namespace xr {
@@ -50,6 +51,56 @@ template <typename T> __device__ __forceinline__ T unpack(const U128& u, int q) 
     if constexpr (IsFp<T>::value) return __longlong_as_double((long long)b);
     else return static_cast<T>(b);
   }
+}
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Programmatic dependent launch (sm_90+): a kernel launched with the
+// programmatic-stream-serialization attribute may start while the previous
+// kernel on the stream drains; every thread waits here (griddepcontrol.wait:
+// the previous grid completed and its memory is visible) before touching
+// global memory, after the CTA's prologue (barrier init).  The trigger lets
+// the NEXT such launch be scheduled as soon as every CTA of this grid has
+// issued it; its CTAs take SM slots as this grid's CTAs exit and sit in their
+// own wait.  Both are no-ops for ordinary launches.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
+// Host: launch `kern` with the programmatic-stream-serialization attribute
+// (every library kernel calls pdl_trigger / pdl_wait before its first global
+// access), or plainly when XR_NO_PDL is set (A/B).
+inline bool pdl_enabled() { return std::getenv("XR_NO_PDL") == nullptr; }
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t dyn, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = dyn;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, args...);
+}
+
+// Per-CTA timeline (profiling only, xr_debug_timeline): when the launch
+// carries a buffer, one thread appends (cta, event, unit, %globaltimer)
+// records: buf[0] = records written (atomic), buf[1] = capacity, then 2 words
+// per record.  A null buffer costs one predicated branch per event.
+enum TlEvent : unsigned { TL_START = 0, TL_UNIT = 1, TL_UNIT_DONE = 2, TL_CONS_END = 3, TL_FOLD = 4, TL_END = 5 };
+__device__ __forceinline__ void tl_event(unsigned long long* tl, unsigned ev, long long unit) {
+  if (tl == nullptr) return;
+  const unsigned long long i = atomicAdd(tl, 1ull);
+  if (i >= tl[1]) return;
+  tl[2 + 2 * i] = ((unsigned long long)blockIdx.x << 40) | ((unsigned long long)ev << 32) |
+                  (unsigned long long)(unsigned)unit;
+  tl[3 + 2 * i] = globaltimer_ns();
 }
 
 // Resident CTAs per SM of kernel KERN at `block` threads and `dyn` bytes of

@@ -371,6 +371,40 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   SegArgs& s = p->seg;
   s.O = O; s.C = C; s.L = L; s.rowStride = rowStride; s.oStride = oStride;
   s.Sr = Sr; s.Sc = Sc; s.units = p->units;
+
+  // Guided units for the whole-array stream (R shape): per-CTA timelines
+  // (tools/timeline.py, r02b) showed the equal-unit tail -- the CTAs finish
+  // over about one unit duration (4 us at 512 MiB, 10 us at 4 GiB) -- plus a
+  // last-CTA fold over 8-9K unit partials.  Phase k gives each of the G
+  // resident CTAs one unit of half the remaining work; once that falls below
+  // two stages the rest goes in one-stage units.
+  if (stream && O == 1 && C == 1 && env.get("XR_STREAM_SPLITS") == nullptr && env.get("XR_NO_GUIDED") == nullptr) {
+    Guided& gd = s.gd;
+    const int64_t G = (int64_t)std::max(num_sms, 1) * 3;      // resident CTAs (64 KiB ring each)
+    const int64_t min_len = std::max<int64_t>(vec, stage_elems);
+    // fp32 '+': each consumer thread owns 16 accumulators, so a unit of len
+    // elements gives chains of len / (kBlock * 16) (<= kChainCap, C9)
+    const int64_t cap_len = chain_capped ? (int64_t)kChainCap * kBlock * 16 : INT64_MAX;
+    int64_t rem = L, c = 0, u = 0;
+    int k = 0;
+    while (k < kMaxPhases - 1) {
+      int64_t len = std::min<int64_t>((rem / 2) / G, cap_len) / vec * vec;
+      if (len < 2 * min_len) break;
+      gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = len;
+      u += G; c += len * G; rem -= len * G; ++k;
+    }
+    const int64_t last = std::min<int64_t>(std::max<int64_t>(min_len, cdiv(cdiv(rem, 4 * G), vec) * vec),
+                                           std::max<int64_t>(vec, cap_len / vec * vec));
+    gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = last;
+    u += cdiv(rem, last);
+    ++k;
+    gd.u0[k] = u; gd.c0[k] = L;
+    gd.nph = k;
+    s.Sr = 1; s.Sc = u; s.units = u;
+    p->splits = u;
+    p->units = u;
+    p->ws_bytes = u * asz;
+  }
 }
 
 }  // namespace xr

@@ -124,6 +124,8 @@ __device__ __forceinline__ int64_t xsplit(int64_t n, int64_t parts, int64_t i) {
 // CTA-wide units, static round robin (deterministic), seg decomposition.
 template <int XF, typename T>
 __global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in2) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using X = Xf<XF, T>;
   using Acc = typename X::Acc;
   using Out = typename X::Out;
@@ -187,6 +189,8 @@ __global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in
 
 template <int XF, typename T>
 __global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const void* in2) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using X = Xf<XF, T>;
   using Out = typename X::Out;
   Out* out = static_cast<Out*>(a.out);
@@ -201,6 +205,8 @@ __global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const vo
 // Column shapes (RK, KRK): CTA-wide column units, static round robin.
 template <int XF, typename T, int VEC>
 __global__ void __launch_bounds__(kBlock) xform_col_kernel(const __grid_constant__ ColArgs a, const void* in2) {
+  pdl_trigger();
+  pdl_wait();  // no global access above this line
   using X = Xf<XF, T>;
   __shared__ __align__(16) unsigned char sm[col_unit_smem<X, VEC>()];
   __shared__ int s_last;
@@ -209,27 +215,28 @@ __global__ void __launch_bounds__(kBlock) xform_col_kernel(const __grid_constant
 }
 
 template <int XF, typename T, int VEC>
-static void xform_col_launch(const ColArgs& c, const void* in2, int sms, cudaStream_t s) {
+static cudaError_t xform_col_launch(const ColArgs& c, const void* in2, int sms, cudaStream_t s) {
   const int occ = occ_dev<xform_col_kernel<XF, T, VEC>>(kBlock, 0);
-  xform_col_kernel<XF, T, VEC><<<(unsigned)grid_for(c.units, sms, occ), kBlock, 0, s>>>(c, in2);
+  return launch_pdl(xform_col_kernel<XF, T, VEC>, dim3((unsigned)grid_for(c.units, sms, occ)), dim3(kBlock), 0, s, c, in2);
 }
 
 template <int XF, typename T>
 static cudaError_t xform_launch(Plan& p, const void* in2, int sms, cudaStream_t s) {
+  cudaError_t le = cudaSuccess;
   if (p.kernel == K_FILL || p.kernel == K_IDENT) {
     EltArgs e = p.elt;
     if (p.kernel == K_FILL) e.in = nullptr;
     const int64_t grid = grid_for((e.n + kBlock - 1) / kBlock, sms, 8);
-    xform_ident_kernel<XF, T><<<(unsigned)grid, kBlock, 0, s>>>(e, in2);
+    le = launch_pdl(xform_ident_kernel<XF, T>, dim3((unsigned)grid), dim3(kBlock), 0, s, e, in2);
   } else if (p.kernel == K_COL) {
-    if (p.vec > 1) xform_col_launch<XF, T, 16 / sizeof(T)>(p.col, in2, sms, s);
-    else xform_col_launch<XF, T, 1>(p.col, in2, sms, s);
+    if (p.vec > 1) le = xform_col_launch<XF, T, 16 / sizeof(T)>(p.col, in2, sms, s);
+    else le = xform_col_launch<XF, T, 1>(p.col, in2, sms, s);
   } else {
     const int occ = occ_dev<xform_kernel<XF, T>>(kBlock, 0);
-    xform_kernel<XF, T><<<(unsigned)grid_for(p.units, sms, occ), kBlock, 0, s>>>(p.seg, in2);
+    le = launch_pdl(xform_kernel<XF, T>, dim3((unsigned)grid_for(p.units, sms, occ)), dim3(kBlock), 0, s, p.seg, in2);
   }
   count_launch();
-  return cudaPeekAtLastError();
+  return le != cudaSuccess ? le : cudaPeekAtLastError();
 }
 
 }  // namespace xr

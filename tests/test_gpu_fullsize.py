@@ -141,8 +141,8 @@ def test_cfg5_op_type_matrix_512cubed(op, dtype):
                                                                        oracle.DTYPES[dtype], mask))
         xd = torch.from_numpy(x).cuda()
         g = gpu_full(op, dtype, dims, lv, xd)
-        if g.size <= 512:
-            check(op, dtype, dims, lv, g, x, exact=(op == "*"))
-        else:
-            sampled_check(op, dtype, dims, lv, x, g, nsamples=96, seed=mask)
+        # every output of every cell against the oracle on the whole nest:
+        # integer / bitwise / logical cells and the exact-regime fp products
+        # are all bit-exact (the 262,144-output masks included; ~2 s each)
+        check(op, dtype, dims, lv, g, x, exact=(op == "*"))
         del xd

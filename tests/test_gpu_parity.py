@@ -11,7 +11,7 @@ import pytest
 import datagen
 from datagen import recipes
 import oracle
-from gpu_util import check, gpu_reduce
+from gpu_util import seg_len, check, gpu_reduce
 
 pytestmark = pytest.mark.gpu
 
@@ -89,9 +89,17 @@ def test_fp_sums_exact_regime(dtype):
 @pytest.mark.parametrize("dtype", ["fp32", "fp64"])
 @pytest.mark.parametrize("kind", ["u01", "um11", "mulgen"])
 def test_fp_general_data(dtype, kind):
+    """General (non-exact) fp data under the C9 / C10 bounds.  Reading C10
+    defines the general-regime product bound on segments of at most 512
+    factors (1 +- 1e-3), so '*' runs only the masks whose segment is <= 512;
+    the (8, 8, 8) and (7, 9, 8) nests give every mask such a segment.  Longer
+    product segments are covered by the exact regime (bit-exact)."""
     op = "*" if kind == "mulgen" else "+"
-    for dims in [(64, 64, 128), (17, 1000, 33)]:
+    shapes = [(64, 64, 128), (17, 1000, 33)] + ([(8, 8, 8), (7, 9, 8)] if op == "*" else [])
+    for dims in shapes:
         for levels in ALL_MASKS:
+            if op == "*" and seg_len(dims, levels) > 512:
+                continue
             x = recipes.make(kind, dims, 7, dtype, 123)
             check(op, dtype, dims, levels, gpu_reduce(op, dtype, dims, levels, x), x)
 

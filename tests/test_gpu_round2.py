@@ -124,14 +124,16 @@ def test_tma_encode_failure_falls_back(monkeypatch):
     got = xr.reduce(xd, "+", "w", nest=dims)
     torch.cuda.synchronize()
     assert xr.xr_launch_count() - n0 == 1
-    assert np.array_equal(got.cpu().numpy(), oracle.reduce("+", "int32", dims, "w", x))
+    assert np.array_equal(got.cpu().numpy().reshape(-1), oracle.reduce("+", "int32", dims, "w", x))
 
 
 @pytest.mark.parametrize("G,skip", [(2, 1), (4, 0), (3, 2)])
 def test_fused_exchange_times_out_without_stale_write(monkeypatch, G, skip):
     """One simulated rank never launches: the others' bounded waits expire,
     they leave out unchanged (no stale combine) and the call reports
-    XR_ERR_NCCL."""
+    XR_ERR_NCCL.  The sim's per-stream warm-up leaves every out
+    at its local sum n_local except rank 0's, restored to the caller's -7; a
+    stale combine of the mailboxes would write (G - 1) * n_local instead."""
     import torch
     import paper_conf_ppopp_xutycc14_b200 as xr
     monkeypatch.setenv("XR_TEST_SIM_SKIP_RANK", str(skip))
@@ -143,7 +145,7 @@ def test_fused_exchange_times_out_without_stale_write(monkeypatch, G, skip):
                                 [xd[r * n_local:(r + 1) * n_local].data_ptr() for r in range(G)],
                                 [o.data_ptr() for o in outs])
     assert st == xr.ERR_NCCL
-    assert [int(o.item()) for o in outs] == [-7] * G
+    assert [int(o.item()) for o in outs] == [-7] + [n_local] * (G - 1)
     monkeypatch.delenv("XR_TEST_SIM_SKIP_RANK")
     st = xr.xr_reduce_fused_sim("+", "int64", (n_local, 1, 1), 7,
                                 [xd[r * n_local:(r + 1) * n_local].data_ptr() for r in range(G)],

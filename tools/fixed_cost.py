@@ -29,6 +29,23 @@ def timeit(fn, reps=25):
     return sorted(a.elapsed_time(b) for a, b in ev)[reps // 2] * 1e3  # us
 
 
+def timeit_b2b(fn, reps=25):
+    """Per-launch time of `reps` back-to-back launches with NO event records
+    between them (events only around the loop): a launch's drain can overlap
+    the next one's start (programmatic dependent launch)."""
+    s = torch.cuda.current_stream()
+    for _ in range(3):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(s)
+    for _ in range(reps):
+        fn()
+    b.record(s)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) * 1e3 / reps
+
+
 def fit(xs, ts):
     A = np.vstack([np.ones(len(xs)), np.array(xs, float)]).T
     (a, b), *_ = np.linalg.lstsq(A, np.array(ts), rcond=None)
@@ -48,6 +65,12 @@ for name, sizes in [("stream-R-fp32", [1 << k for k in range(24, 31)])]:
     a, bw = fit(xs[2:], ts[2:])  # >= 64 MiB (past L2)
     print(json.dumps({"series": name, "label": label, "sizes_bytes": xs, "us": [round(t, 2) for t in ts],
                       "fixed_us": round(a, 2), "stream_GBps": round(bw, 1)}), flush=True)
+    ts = [timeit_b2b(lambda: xr.xr_reduce("+", "fp32", (n, 1, 1), "gwv", big.data_ptr(), out.data_ptr(), sh))
+          for n in sizes]
+    a, bw = fit(xs[2:], ts[2:])
+    print(json.dumps({"series": name + "-back-to-back", "label": label, "sizes_bytes": xs,
+                      "us": [round(t, 2) for t in ts], "fixed_us": round(a, 2), "stream_GBps": round(bw, 1)}),
+          flush=True)
 # reference series: torch's own copy (the MEASURED_PEAKS kernel) and torch.sum
 for name, mk in [("torch-copy", lambda n: (lambda d=torch.empty(n, device="cuda"): d.copy_(big[:n]))),
                  ("torch-sum", lambda n: (lambda: torch.sum(big[:n])))]:

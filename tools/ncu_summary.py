@@ -1,7 +1,7 @@
 #!/usr/bin/env python3
 """Summarise ncu reports (gpurun_out/ncu/<case>_<TAG>.ncu-rep) into profiles/.
 
-  python tools/ncu_summary.py TAG [--launches CSV]
+  python tools/ncu_summary.py TAG [--launches CSV] [--outdir DIR]
 
 <case> is a tools/kdriver.py case name (cfg2-f32-sum, cfg3-col, cfg4-heat,
 cfg5-<op>-<dtype>-<mask>, nest-..., mc-pi-N, ...).  Writes
@@ -92,10 +92,22 @@ def raw(rep):
 
 def main():
     tag = sys.argv[1]
+    # --outdir D: write the summary and the merged json files to D instead of
+    # profiles/ (used ON the GPU box, where the .ncu-rep files are too large
+    # to bring back; the caller copies D into profiles/)
+    outdir = os.path.join(ROOT, "profiles")
+    if "--outdir" in sys.argv:
+        outdir = sys.argv[sys.argv.index("--outdir") + 1]
+        for f in ("ncu_traffic.json", "ncu_dram.json"):
+            src = os.path.join(ROOT, "profiles", f)
+            if os.path.exists(src) and not os.path.exists(os.path.join(outdir, f)):
+                os.makedirs(outdir, exist_ok=True)
+                with open(src) as a, open(os.path.join(outdir, f), "w") as b:
+                    b.write(a.read())
     reps = sorted(glob.glob(os.path.join(ROOT, "gpurun_out", "ncu", f"*_{tag}.ncu-rep")))
-    os.makedirs(os.path.join(ROOT, "profiles"), exist_ok=True)
-    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    dpath = os.path.join(ROOT, "profiles", "ncu_dram.json")
+    os.makedirs(outdir, exist_ok=True)
+    tpath = os.path.join(outdir, "ncu_traffic.json")
+    dpath = os.path.join(outdir, "ncu_dram.json")
     traffic = json.load(open(tpath)) if os.path.exists(tpath) else {}
     dram = json.load(open(dpath)) if os.path.exists(dpath) else {}
     lines = [f"# ncu summary — {tag}", "",
@@ -145,9 +157,9 @@ def main():
             dram[WORKLOAD[case]] = rec
             traffic[WORKLOAD[case]] = rd + wr
         traffic[f"{case}@{tag}"] = rd + wr
-    if len(sys.argv) > 3 and sys.argv[2] == "--launches":
-        src = sys.argv[3]
-        dst = os.path.join(ROOT, "profiles", f"launches_{tag}.csv")
+    if "--launches" in sys.argv:
+        src = sys.argv[sys.argv.index("--launches") + 1]
+        dst = os.path.join(outdir, f"launches_{tag}.csv")
         with open(src) as f, open(dst, "w") as g:
             g.write("".join(l for l in f if not l.startswith("==")))
         # share of the step per kernel name
@@ -162,7 +174,7 @@ def main():
         for k, v in sorted(tot.items(), key=lambda kv: -kv[1]):
             n = sum(1 for r in rows if r["Kernel Name"] == k)
             lines.append(f"| `{k[:70]}` | {n} | {v:.0f} | {v / s:.4f} |")
-    with open(os.path.join(ROOT, "profiles", f"ncu_{tag}.md"), "w") as f:
+    with open(os.path.join(outdir, f"ncu_{tag}.md"), "w") as f:
         f.write("\n".join(lines) + "\n")
     json.dump(traffic, open(tpath, "w"), indent=1, sort_keys=True)
     json.dump(dram, open(dpath, "w"), indent=1, sort_keys=True)
