@@ -37,12 +37,12 @@ struct ExchArgs {
                                             // (host-mapped: readable without a device sync)
 };
 
-// Guided unit schedule of the stream kernel's whole-array (R) shape: phase k
-// holds units [u0[k], u0[k+1]) of len[k] elements each, starting at element
-// c0[k] (the last unit of a phase ends at c0[k+1]).  Early phases hand every
-// CTA a long unit (half the remaining work per phase), the last phase short
-// ones, so the CTAs finish within about one short unit of each other while
-// the number of unit partials (and the last CTA's fold) stays small.
+// Guided unit schedule of the stream kernel's whole-array (R) shape (opt-in,
+// XR_GUIDED=1; xr_plan.cpp has the measurements): phase k holds units
+// [u0[k], u0[k+1]) of len[k] elements each, starting at element c0[k] (the
+// last unit of a phase ends at c0[k+1]).  Phase 0 keeps the equal units, the
+// later phases halve the unit length so the CTAs finish within about one
+// short unit of each other.
 constexpr int kMaxPhases = 12;
 struct Guided {
   int nph;                       // 0: equal units (Sr x Sc split)

@@ -473,10 +473,20 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
       tl_event(a.tl, TL_START, 0);
       int64_t g = 0;
       int seq = 0;
+      // claims run two units ahead when units are short (guided tail phases
+      // of one or two stages): a claim's L2 round trip then overlaps two
+      // units' streaming instead of stalling the ring
+      const bool deep = a.gd.nph > 1;
       long long u = claim_first(a.sched);
+      long long n1 = deep ? claim_next(a.sched) : 0;
       while (true) {
         tl_event(a.tl, TL_UNIT, u);
-        const long long nu = claim_next(a.sched);  // next claim, in flight
+        long long nu = claim_next(a.sched);  // next claim, in flight
+        if (deep) {
+          const long long t = n1;
+          n1 = nu;
+          nu = t;
+        }
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < a.units ? u : -1;
         ++seq;

@@ -373,31 +373,50 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   s.Sr = Sr; s.Sc = Sc; s.units = p->units;
 
   // Guided units for the whole-array stream (R shape): per-CTA timelines
-  // (tools/timeline.py, r02b) showed the equal-unit tail -- the CTAs finish
-  // over about one unit duration (4 us at 512 MiB, 10 us at 4 GiB) -- plus a
-  // last-CTA fold over 8-9K unit partials.  Phase k gives each of the G
-  // resident CTAs one unit of half the remaining work; once that falls below
-  // two stages the rest goes in one-stage units.
-  if (stream && O == 1 && C == 1 && env.get("XR_STREAM_SPLITS") == nullptr && env.get("XR_NO_GUIDED") == nullptr) {
+  // (tools/timeline.py) showed the equal-unit tail -- the CTAs finish over
+  // about one unit duration (4 us at 512 MiB, 10 us at 4 GiB).  The per-CTA
+  // rate varies by up to 1.6x under full load, so a unit may only be as long
+  // as the work still queued behind it can cover: phase 0 keeps the equal
+  // units (u0 = L / S) for all but the last R = 2 G u0 elements; phase k then
+  // hands out 2G units of u0 / 2^k (half the remaining work), so the queued
+  // work stays two fair-share unit durations ahead of every claim, down to
+  // two-stage units.  (A first version started at half the array in G units,
+  // "factoring": a slow CTA's first unit outlasted the rest by 60 us, r02c.)
+  // MEASURED NEUTRAL (r02d / perf3 A/B on one box: 512 MiB 84.4 vs 84.5 us,
+  // 4 GiB 583-588 vs 582-588 us, back-to-back within 0.5 us): the tail
+  // shrinks from 4-10 us to 1.3-1.7 us but the short units' per-unit cost
+  // (claim round trip, consumer epilogue) gives it back, so equal units stay
+  // the default; XR_GUIDED=1 selects this schedule.
+  if (stream && O == 1 && C == 1 && env.get("XR_STREAM_SPLITS") == nullptr && env.get("XR_GUIDED") != nullptr) {
     Guided& gd = s.gd;
     const int64_t G = (int64_t)std::max(num_sms, 1) * 3;      // resident CTAs (64 KiB ring each)
-    const int64_t min_len = std::max<int64_t>(vec, stage_elems);
-    // fp32 '+': each consumer thread owns 16 accumulators, so a unit of len
-    // elements gives chains of len / (kBlock * 16) (<= kChainCap, C9)
-    const int64_t cap_len = chain_capped ? (int64_t)kChainCap * kBlock * 16 : INT64_MAX;
-    int64_t rem = L, c = 0, u = 0;
+    const char* gm = env.get("XR_GUIDED_MIN_BYTES");  // tuning override (default: two stages)
+    const int64_t min_len = std::max<int64_t>(vec, (gm ? std::max(16ll, std::atoll(gm)) : 2ll * kStageBytes) / size);
+    const int64_t u0 = std::max<int64_t>(min_len, cdiv(cdiv(L, std::max<int64_t>(Sc, 1)), vec) * vec);
+    const int64_t bulk = L > 2 * G * u0 ? (L - 2 * G * u0) / vec * vec : 0;  // phase boundaries stay 16-B aligned
+    int64_t rem = L - bulk, c = 0, u = 0;
     int k = 0;
-    while (k < kMaxPhases - 1) {
-      int64_t len = std::min<int64_t>((rem / 2) / G, cap_len) / vec * vec;
-      if (len < 2 * min_len) break;
-      gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = len;
-      u += G; c += len * G; rem -= len * G; ++k;
+    if (bulk > 0) {  // phase 0: equal units over the bulk of the array
+      gd.u0[k] = 0; gd.c0[k] = 0; gd.len[k] = u0;
+      u = cdiv(bulk, u0);
+      c = bulk;
+      ++k;
+      // the last phase-0 unit may be short: phase 1 starts right after it
     }
-    const int64_t last = std::min<int64_t>(std::max<int64_t>(min_len, cdiv(cdiv(rem, 4 * G), vec) * vec),
-                                           std::max<int64_t>(vec, cap_len / vec * vec));
-    gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = last;
-    u += cdiv(rem, last);
-    ++k;
+    int64_t len = u0 / 2 / vec * vec;
+    while (k < kMaxPhases - 1 && len >= 2 * min_len && rem > 0) {
+      int64_t part = std::max<int64_t>(rem / 2 / vec * vec, len);
+      if (part >= rem - min_len) part = rem;
+      gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = len;
+      u += cdiv(part, len); c += part; rem -= part; ++k;
+      len = len / 2 / vec * vec;
+    }
+    if (rem > 0) {
+      gd.u0[k] = u; gd.c0[k] = c; gd.len[k] = min_len;
+      u += cdiv(rem, min_len);
+      c += rem;
+      ++k;
+    }
     gd.u0[k] = u; gd.c0[k] = L;
     gd.nph = k;
     s.Sr = 1; s.Sc = u; s.units = u;
