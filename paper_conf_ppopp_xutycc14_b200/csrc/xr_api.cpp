@@ -466,6 +466,7 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   if (p.kernel == K_STREAM || p.kernel == K_COLTMA || p.kernel == K_ROWS || p.kernel == K_RKR) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
+  if (p.kernel == K_COLSMALL) ctas = (p.units + kBlock / 32 - 1) / (kBlock / 32);
   info->grid = p.kernel == K_NONE ? 0 : grid_for(ctas, num_sms, kTargetCtasPerSm);
   if (p.grid_hint > 0) info->grid = std::min(info->grid, p.grid_hint);
   info->ws_bytes = p.ws_bytes;

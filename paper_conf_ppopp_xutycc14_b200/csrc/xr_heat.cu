@@ -56,8 +56,8 @@ __device__ __forceinline__ double ld_row(const double* p) { return __ldg(p); }
 // peak in profiles/ r01).
 template <int VEC>
 __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP_MAX, double>;
   constexpr int NW = kBlock / 32;
   constexpr int STRIP = 32 * VEC;
@@ -193,8 +193,8 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   if (warp == 0) {
     // producer warp: row q of the tile into slot q % kHeatSlots once the
     // consumers released the row kHeatSlots earlier
@@ -311,8 +311,8 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
       int64_t q = 0;  // global row counter (slot = q % kHeatSlots)

@@ -269,8 +269,8 @@ template <int OP, typename T, int W, int BLOCK, int U>
 #define XR_SEG_MINB 4
 #endif
 __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_constant__ SegArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   __shared__ Acc smem[32];
@@ -281,12 +281,15 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
 
   if constexpr (W == BLOCK) {
     __shared__ long long s_unit[2];
-    if (threadIdx.x == 0) s_unit[0] = claim_first(a.sched);
+    // one unit per CTA (small, latency-bound inputs): static assignment, no
+    // claim round trip at the start and no exit counter at the end
+    const bool one_each = a.units <= (int64_t)gridDim.x;
+    if (threadIdx.x == 0) s_unit[0] = one_each ? (long long)blockIdx.x : claim_first(a.sched);
     __syncthreads();
     long long u = s_unit[0];
     int par = 1;
     while (u < a.units) {
-      if (threadIdx.x == 0) s_unit[par] = claim_next(a.sched);  // next, in flight
+      if (threadIdx.x == 0) s_unit[par] = one_each ? (long long)a.units : claim_next(a.sched);  // next, in flight
       int64_t o;
       Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
       v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
@@ -319,7 +322,7 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
       u = s_unit[par];
       par ^= 1;
     }
-    sched_exit(a.sched);
+    if (!one_each) sched_exit(a.sched);
   } else {
     static_assert(W <= 32 && (32 % W) == 0, "sub-warp group");
     const int lane = threadIdx.x & (W - 1);
@@ -462,8 +465,8 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
 
   if (warp == 0) {
     // ---------------- producer warp: claims units, publishes their ids and
@@ -697,8 +700,8 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
 
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
@@ -796,8 +799,8 @@ __global__ void __launch_bounds__(kWsBlock) rows_kernel(SegArgs a) {
 // paper's 2^20 x 2 x 32 gang case).
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __grid_constant__ ColArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int VEC = 16 / sizeof(T);
@@ -1010,8 +1013,8 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
 
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
@@ -1174,6 +1177,73 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   }
 }
 
+// ------------------------------------------------------------- small column kernel
+// RK / KRK on SMALL inputs (latency bound, e.g. the paper-style testsuite nest
+// 64 x 64 x 128 at gang or worker level) with few reduced rows (R <= 256):
+// one WARP per group of CW = 32 B of kept columns; lane l folds rows l, l+32,
+// ... (two 16-B loads per row, four in flight), then one warp reduction per
+// column (a2: REDUX / shuffles) and lanes 0..CW-1 write the CW outputs.  No
+// shared memory, no barrier and no gang tier, and 8x more CTAs than the
+// CTA-per-tile column kernels (r01: 64 CTAs of 32 KiB for cfg1 G / W, 5.3 us
+// graph-replayed, vs 2.1 us for the 512-CTA row case).
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) colsmall_kernel(const __grid_constant__ ColArgs a) {
+  pdl_wait();  // no global access above this line
+  pdl_trigger();
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  constexpr int CW = 2 * VEC;  // columns per warp
+  const int lane = threadIdx.x & 31;
+  const int64_t gw = ((int64_t)blockIdx.x * kBlock + threadIdx.x) >> 5;
+  if (gw >= a.units) return;  // warp-uniform
+  const int64_t b = gw / a.tiles, c0 = (gw - b * a.tiles) * CW;
+  const bool two = c0 + CW <= a.K;  // else only the first vector (K % VEC == 0)
+  const T* __restrict__ base = static_cast<const T*>(a.in) + b * a.R * a.K + c0;
+  T* out = static_cast<T*>(a.out);
+  Acc acc[CW];
+#pragma unroll
+  for (int q = 0; q < CW; ++q) acc[q] = O::identity();
+  int64_t r = lane;
+  for (; r + 32 < a.R; r += 64) {  // two rows, four 16-B loads in flight
+    const T* p0 = base + r * a.K;
+    const T* p1 = p0 + 32 * a.K;
+    const U128 x0 = ld_stream(p0), x2 = ld_stream(p1);
+    U128 x1 = x0, x3 = x2;
+    if (two) { x1 = ld_stream(p0 + VEC); x3 = ld_stream(p1 + VEC); }
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) {
+      acc[q] = O::combine(acc[q], O::lift(unpack<T>(x0, q)));
+      acc[q] = O::combine(acc[q], O::lift(unpack<T>(x2, q)));
+      if (two) {
+        acc[VEC + q] = O::combine(acc[VEC + q], O::lift(unpack<T>(x1, q)));
+        acc[VEC + q] = O::combine(acc[VEC + q], O::lift(unpack<T>(x3, q)));
+      }
+    }
+  }
+  if (r < a.R) {
+    const T* p0 = base + r * a.K;
+    const U128 x0 = ld_stream(p0);
+    U128 x1 = x0;
+    if (two) x1 = ld_stream(p0 + VEC);
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) {
+      acc[q] = O::combine(acc[q], O::lift(unpack<T>(x0, q)));
+      if (two) acc[VEC + q] = O::combine(acc[VEC + q], O::lift(unpack<T>(x1, q)));
+    }
+  }
+  Acc mine = O::identity();
+#pragma unroll
+  for (int q = 0; q < CW; ++q) {
+    const Acc v = group_reduce<OP, T, 32>(acc[q]);
+    if (lane == q) mine = v;
+  }
+  if (lane < (two ? CW : VEC)) {
+    const int64_t o = b * a.K + c0 + lane;
+    out[o] = merge_init<OP, T>(mine, out, o, a.init_from_out);
+  }
+}
+
 // ------------------------------------------------------------- col kernel
 // Lanes own VEC contiguous kept columns (a 32*VEC-column tile per warp row);
 // the CTA's warps stride over the reduced rows of a row chunk; the worker tier
@@ -1184,8 +1254,8 @@ template <int OP, typename T, int VEC, int BLOCK, int U>
 #define XR_COL_MINB 1
 #endif
 __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_constant__ ColArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int NW = BLOCK / 32;
@@ -1352,8 +1422,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     fence_mbar_init();
   }
   __syncthreads();
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
 
   if (warp == 0) {
     // ---------------- producer warp
@@ -1529,8 +1599,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
 // ------------------------------------------------------------- elementwise
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   const T* in = static_cast<const T*>(a.in);
   T* out = static_cast<T*>(a.out);
@@ -1540,8 +1610,8 @@ __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
 
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) fill_kernel(EltArgs a) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   T* out = static_cast<T*>(a.out);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (int64_t)gridDim.x * blockDim.x)
@@ -1551,8 +1621,8 @@ __global__ void __launch_bounds__(kBlock) fill_kernel(EltArgs a) {
 // Fixed rank-order combine of gathered partial results (sharded path).
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int nranks, int64_t n, T* out) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using O = Op<OP, T>;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     typename O::Acc v = O::identity();
@@ -1619,6 +1689,11 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.seg)) return e;
+      break;
+    }
+    case K_COLSMALL: {
+      const int64_t grid = (p.units + kBlock / 32 - 1) / (kBlock / 32);
+      if (cudaError_t e = launch_pdl(colsmall_kernel<OP, T>, dim3((unsigned)grid), dim3(kBlock), 0, s, p.col)) return e;
       break;
     }
     case K_COLFLAT: {

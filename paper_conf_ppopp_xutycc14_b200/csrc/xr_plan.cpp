@@ -138,6 +138,23 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const int cv = aligned ? vec : 1;
     // seg_only (the fused multi-input / multi-variable launches): always the
     // register column decomposition below (their col_unit, xr_colunit.cuh)
+    // Small inputs with few reduced rows: one warp per 32 B of kept columns
+    // (colsmall_kernel), no gang tier -- the latency-bound testsuite nest.
+    {
+      const int64_t cw = 2 * vec;
+      const int64_t groups = B * cdiv(K, cw);
+      if (!seg_only && seg_only_small && aligned && R <= 256 && groups >= 256 &&
+          env.get("XR_NO_COLSMALL") == nullptr) {
+        p->kernel = K_COLSMALL;
+        p->vec = vec;
+        p->splits = 1;
+        p->units = groups;  // warps
+        p->group = 32;
+        ColArgs& c = p->col;
+        c.B = B; c.R = R; c.K = K; c.tiles = cdiv(K, cw); c.S = 1; c.units = groups;
+        return;
+      }
+    }
     // Narrow rows (power-of-two row_bytes in [16, 512] B, or up to 4 KiB for
     // small inputs): the flat column kernel streams whole rows contiguously.
     const int64_t row_bytes = K * size;

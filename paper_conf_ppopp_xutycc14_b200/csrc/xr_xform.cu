@@ -124,8 +124,8 @@ __device__ __forceinline__ int64_t xsplit(int64_t n, int64_t parts, int64_t i) {
 // CTA-wide units, static round robin (deterministic), seg decomposition.
 template <int XF, typename T>
 __global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in2) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using X = Xf<XF, T>;
   using Acc = typename X::Acc;
   using Out = typename X::Out;
@@ -189,8 +189,8 @@ __global__ void __launch_bounds__(kBlock) xform_kernel(SegArgs a, const void* in
 
 template <int XF, typename T>
 __global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const void* in2) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using X = Xf<XF, T>;
   using Out = typename X::Out;
   Out* out = static_cast<Out*>(a.out);
@@ -205,8 +205,8 @@ __global__ void __launch_bounds__(kBlock) xform_ident_kernel(EltArgs a, const vo
 // Column shapes (RK, KRK): CTA-wide column units, static round robin.
 template <int XF, typename T, int VEC>
 __global__ void __launch_bounds__(kBlock) xform_col_kernel(const __grid_constant__ ColArgs a, const void* in2) {
-  pdl_trigger();
   pdl_wait();  // no global access above this line
+  pdl_trigger();
   using X = Xf<XF, T>;
   __shared__ __align__(16) unsigned char sm[col_unit_smem<X, VEC>()];
   __shared__ int s_last;

@@ -17,7 +17,7 @@ import pytest
 import datagen
 import oracle
 from datagen import recipes
-from gpu_util import check, torch_dt
+from gpu_util import check, gpu_reduce, torch_dt
 
 pytestmark = pytest.mark.gpu
 MASKS = ["g", "w", "v", "gw", "gv", "wv", "gwv"]
@@ -165,3 +165,23 @@ def test_python_binding_validates_device_calls():
         xr.reduce(x, "+", "g", nest=(2, 3, 4), out=torch.zeros(12, dtype=torch.int32))  # host out
     got = xr.reduce(x.reshape(2, 3, 2, 2), "+", "g")              # 4-D: leading dims flattened -> (6, 2, 2)
     assert got.cpu().tolist() == [[sum(range(k, 24, 4)) for k in range(j * 2, j * 2 + 2)] for j in range(2)]
+
+
+@pytest.mark.parametrize("op,dtype", [("+", "int32"), ("+", "fp32"), ("*", "int64"), ("max", "fp64"),
+                                      ("^", "int32"), ("&&", "fp32"), ("min", "int64"), ("||", "int32")])
+def test_colsmall_kernel(op, dtype):
+    """Small column shapes with few reduced rows (the cfg1 testsuite nest at
+    gang / worker level): one warp per 32 B of kept columns, rows strided by
+    lane (ragged R), a half-width last group (K % (2 VEC) != 0), batches, init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    vec = 16 // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    cases = [((64, 64, 128), "g"), ((64, 64, 128), "w"), ((3, 601 * vec, 1), "g"),
+             ((256, 515 * vec, 1), "g"), ((40, 33, 24 * vec + vec), "w"), ((7, 2, 300 * vec), "w"),
+             ((31, 1, 2048 * vec), "g"), ((2, 65, 1024 * vec), "w")]
+    for dims, lv in cases:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, sum(dims) + 1)
+        plan = xr.xr_plan_describe(op, dtype, dims, lv, 256)
+        assert plan["kernel"] == "colsmall", (dims, lv, plan)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 5)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)

@@ -9,7 +9,7 @@ import paper_conf_ppopp_xutycc14_b200 as xr  # noqa: E402
 dims = (64, 64, 128)
 x = torch.randint(-1000, 1000, (64 * 64 * 128,), dtype=torch.int32, device="cuda")
 s = torch.cuda.Stream()
-for lv in ["g", "w", "v", "gwv"]:
+for lv in ["g", "w", "v", "gw", "gv", "wv", "gwv"]:
     o = torch.zeros(xr.xr_out_count(dims, lv), dtype=torch.int32, device="cuda")
     with torch.cuda.stream(s):
         xr.xr_reserve("+", "int32", dims, lv, s.cuda_stream)
