@@ -311,7 +311,14 @@ int xr_heat_run(int64_t nj, int64_t ni, int64_t iters, double* T1, double* T2,
  * row n_local (both halos are unused at the global boundary). */
 int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* T2,
                          double* residual, xr_comm_t comm, xr_stream_t stream);
-/* iters steps swapping T1/T2 (residuals: DEVICE, iters fp64). */
+/* iters steps swapping T1/T2 (residuals: DEVICE, iters fp64), overlapped:
+ * each sweep computes its two boundary rows first, the halo exchange of those
+ * rows runs on the communicator's internal stream while the interior rows
+ * sweep, and the residual allreduce of sweep k is issued after the halos of
+ * sweep k+1 (one sweep late, hidden behind the next interior sweep).  When the
+ * work enqueued on `stream` completes, every residuals[k] is final and
+ * bit-identical to the serial xr_heat_step_sharded sequence (max is exact);
+ * only a host that polled residuals[k] mid-run would see it one sweep late. */
 int xr_heat_run_sharded(int64_t n_local, int64_t ni, int64_t iters, double* T1, double* T2,
                         double* residuals, xr_comm_t comm, xr_stream_t stream);
 /* Single-device simulation of the same protocol over nranks slabs (halo

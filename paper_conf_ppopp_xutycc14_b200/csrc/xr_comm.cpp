@@ -22,7 +22,7 @@ int reduce_device_checked(int op, int dtype, const int64_t* dims, unsigned mask,
 cudaError_t gather_combine(int op, int dtype, const void* g, int nranks, int64_t n, void* out, cudaStream_t s);
 int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* je);
 int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
-                   double* residual, cudaStream_t s);
+                   double* residual, cudaStream_t s, const double* res_init = nullptr);
 int reduce_host_into(int op, int dtype, const int64_t* dims, unsigned mask, const void* in_host, void* out_dev,
                      cudaStream_t s);
 }  // namespace xr
@@ -38,6 +38,11 @@ struct xr_comm_s {
   size_t scratch_bytes = 0;
   void* hout = nullptr;     // device copy of the output of xr_reduce_sharded_host
   size_t hout_bytes = 0;
+  // overlapped sharded heat run: a communication stream, its events and the
+  // boundary-row residual slot
+  cudaStream_t cstream = nullptr;
+  cudaEvent_t ev_start = nullptr, ev_bound = nullptr, ev_sweep = nullptr, ev_halo = nullptr, ev_end = nullptr;
+  double* res_bound = nullptr;
   // fused exchange (peer mailboxes over NVLink via CUDA IPC)
   bool fused = false;                         // set up and enabled
   unsigned long long* mailbox = nullptr;      // mine
@@ -206,6 +211,10 @@ int xr_comm_destroy(xr_comm_t comm) {
   if (comm->status) cudaFreeHost(comm->status);
   if (comm->scratch) cudaFree(comm->scratch);
   if (comm->hout) cudaFree(comm->hout);
+  if (comm->res_bound) cudaFree(comm->res_bound);
+  for (cudaEvent_t e : {comm->ev_start, comm->ev_bound, comm->ev_sweep, comm->ev_halo, comm->ev_end})
+    if (e) cudaEventDestroy(e);
+  if (comm->cstream) cudaStreamDestroy(comm->cstream);
   if (comm->nccl && ncclCommDestroy(comm->nccl) != ncclSuccess) st = XR_ERR_NCCL;
   delete comm;
   return st;
@@ -369,18 +378,86 @@ int xr_heat_step_sharded(int64_t n_local, int64_t ni, const double* T1, double* 
   return XR_OK;
 }
 
+// The halo rows of sweep k+1 depend only on the BOUNDARY rows of sweep k, so
+// those are swept first (two one-row launches), the halo exchange runs on a
+// communication stream while the interior sweeps, and the residual allreduce
+// of sweep k is issued on that stream after the halos of sweep k+1: it is
+// lagged one sweep and hidden behind the next interior sweep (SURVEY 8(e),
+// "heat at G = 8").  Every residual is still exact and final when the run
+// returns to the stream: max is exact, and the interior launch merges the
+// boundary rows' maximum (res_init), so residuals are bit-identical to the
+// serial protocol.
+static int halo_exchange(xr_comm_t comm, int64_t n_local, int64_t ni, double* T, cudaStream_t c) {
+  const int r = comm->rank;
+  const bool force = comm->nranks == 1 && std::getenv("XR_FORCE_COLL") != nullptr;
+  const int up = r > 0 ? r - 1 : (force ? r : -1);
+  const int down = r < comm->nranks - 1 ? r + 1 : (force ? r : -1);
+  if (up < 0 && down < 0) return XR_OK;
+  if (ncclGroupStart() != ncclSuccess) return XR_ERR_NCCL;
+  if (up >= 0) {
+    ncclSend(T + ni, (size_t)ni, ncclFloat64, up, comm->nccl, c);
+    ncclRecv(T, (size_t)ni, ncclFloat64, up, comm->nccl, c);
+  }
+  if (down >= 0) {
+    ncclSend(T + n_local * ni, (size_t)ni, ncclFloat64, down, comm->nccl, c);
+    ncclRecv(T + (n_local + 1) * ni, (size_t)ni, ncclFloat64, down, comm->nccl, c);
+  }
+  return ncclGroupEnd() == ncclSuccess ? XR_OK : XR_ERR_NCCL;
+}
+
 int xr_heat_run_sharded(int64_t n_local, int64_t ni, int64_t iters, double* T1, double* T2, double* residuals,
                         xr_comm_t comm, xr_stream_t stream) {
-  if (iters < 0 || (iters > 0 && !residuals)) return XR_ERR_INVALID;
+  if (!comm || n_local < 1 || ni < 0 || !T1 || !T2 || iters < 0 || (iters > 0 && !residuals)) return XR_ERR_INVALID;
+  if (iters == 0) return XR_OK;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (!comm->cstream) {
+    if (cudaStreamCreateWithFlags(&comm->cstream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaMalloc(&comm->res_bound, 2 * sizeof(double)) != cudaSuccess) {
+      cudaGetLastError();
+      return XR_ERR_CUDA;
+    }
+    for (cudaEvent_t* e : {&comm->ev_start, &comm->ev_bound, &comm->ev_sweep, &comm->ev_halo, &comm->ev_end})
+      if (cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) { cudaGetLastError(); return XR_ERR_CUDA; }
+  }
+  cudaStream_t c = comm->cstream;
+  int64_t jb, je;
+  int st = heat_slab_rows(n_local, comm->nranks, comm->rank, &jb, &je);
+  if (st) return st;
+  const int64_t nj = n_local + 2;
+  const bool split = je - jb >= 3;  // boundary rows jb and je-1 swept before the interior
+  auto cu = [](cudaError_t e) { return e == cudaSuccess ? XR_OK : (cudaGetLastError(), XR_ERR_CUDA); };
+  // the communication stream starts after the caller's prior work on `stream`
+  if ((st = cu(cudaEventRecord(comm->ev_start, s))) || (st = cu(cudaStreamWaitEvent(c, comm->ev_start, 0)))) return st;
   double* a = T1;
   double* b = T2;
   for (int64_t it = 0; it < iters; ++it) {
-    int st = xr_heat_step_sharded(n_local, ni, a, b, residuals + it, comm, stream);
-    if (st) return st;
+    if (it > 0 && (st = cu(cudaStreamWaitEvent(s, comm->ev_halo, 0)))) return st;  // a's halos landed
+    if (split) {
+      if ((st = heat_step_rows(nj, ni, jb, jb + 1, a, b, comm->res_bound, s))) return st;
+      if ((st = heat_step_rows(nj, ni, je - 1, je, a, b, comm->res_bound, s, comm->res_bound))) return st;
+      if ((st = cu(cudaEventRecord(comm->ev_bound, s)))) return st;
+      if ((st = heat_step_rows(nj, ni, jb + 1, je - 1, a, b, residuals + it, s, comm->res_bound))) return st;
+    } else {
+      if ((st = heat_step_rows(nj, ni, jb, je, a, b, residuals + it, s))) return st;
+      if ((st = cu(cudaEventRecord(comm->ev_bound, s)))) return st;
+    }
+    // communication stream: b's halos (its boundary rows are final), then the
+    // residual of the PREVIOUS sweep (its interior launch precedes ev_bound)
+    if ((st = cu(cudaStreamWaitEvent(c, comm->ev_bound, 0)))) return st;
+    if ((st = halo_exchange(comm, n_local, ni, b, c))) return st;
+    if ((st = cu(cudaEventRecord(comm->ev_halo, c)))) return st;
+    if (it > 0 && ncclAllReduce(residuals + it - 1, residuals + it - 1, 1, ncclFloat64, ncclMax, comm->nccl, c) !=
+                      ncclSuccess)
+      return XR_ERR_NCCL;
     double* t = a;
     a = b;
     b = t;
   }
+  // the last residual, then join the communication stream back into `stream`
+  if ((st = cu(cudaEventRecord(comm->ev_sweep, s))) || (st = cu(cudaStreamWaitEvent(c, comm->ev_sweep, 0)))) return st;
+  if (ncclAllReduce(residuals + iters - 1, residuals + iters - 1, 1, ncclFloat64, ncclMax, comm->nccl, c) != ncclSuccess)
+    return XR_ERR_NCCL;
+  if ((st = cu(cudaEventRecord(comm->ev_end, c))) || (st = cu(cudaStreamWaitEvent(s, comm->ev_end, 0)))) return st;
   return XR_OK;
 }
 

@@ -40,6 +40,7 @@ struct HeatArgs {
   int64_t jb, je;  // output rows [jb, je) of the buffer (single GPU: [1, nj-1))
   int64_t rows;    // output rows per CTA (bulk kernel: sized for one full wave)
   int64_t ntiles;  // CTAs in the grid
+  const double* res_init;  // non-null: *residual = max(*res_init, this sweep's max) (split sweeps)
 };
 
 __device__ __forceinline__ double stencil(double up, double down, double left, double right) {
@@ -147,7 +148,7 @@ __global__ void __launch_bounds__(kBlock) heat_kernel(HeatArgs a) {
     for (int64_t k = threadIdx.x; k < a.ntiles; k += kBlock) w = O::combine(w, ld_partial(a.partials + k));
     w = block_reduce<OP_MAX, double, kBlock>(w, smem);
     if (threadIdx.x == 0) {
-      *a.residual = w;
+      *a.residual = a.res_init ? O::combine(*a.res_init, w) : w;
       *a.tickets = 0u;
     }
   }
@@ -261,7 +262,7 @@ __global__ void __launch_bounds__(kWsBlock) heat_bulk_kernel(HeatArgs a) {
     for (int64_t k = tid; k < a.ntiles; k += kConsThreads) w = O::combine(w, ld_partial(a.partials + k));
     w = cons_reduce<OP_MAX, double>(w, smem, cw, lane);
     if (tid == 0) {
-      *a.residual = w;
+      *a.residual = a.res_init ? O::combine(*a.res_init, w) : w;
       *a.tickets = 0u;
     }
   }
@@ -436,7 +437,7 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
     for (int64_t k = tid; k < gridDim.x; k += kConsThreads) w = O::combine(w, ld_partial(a.partials + k));
     w = cons_reduce<OP_MAX, double>(w, smem, cw, lane);
     if (tid == 0) {
-      *a.residual = w;
+      *a.residual = a.res_init ? O::combine(*a.res_init, w) : w;
       *a.tickets = 0u;
     }
   }
@@ -444,7 +445,7 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
 
 // Sweep output rows [jb, je) of an nj x ni buffer (rows jb-1 and je are read).
 static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
-                       double* residual, cudaStream_t s) {
+                       double* residual, cudaStream_t s, const double* res_init = nullptr) {
   const bool al16 = ((uintptr_t)T1 % 16 == 0) && ((uintptr_t)T2 % 16 == 0);
   const bool v2 = (ni % 2 == 0) && al16;
   // odd ni: only the persistent kernel stages rows with a per-row 8-B shift
@@ -471,6 +472,7 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
   HeatArgs a;
   a.rows = rows;
   a.T1 = T1; a.T2 = T2; a.residual = residual; a.nj = nj; a.ni = ni; a.ntiles = gx * gy;
+  a.res_init = res_init;
   a.jb = jb; a.je = je;
   void* partials = nullptr;
   unsigned* tickets = nullptr;
@@ -520,8 +522,8 @@ int heat_slab_rows(int64_t n_local, int nranks, int rank, int64_t* jb, int64_t* 
 }
 
 int heat_step_rows(int64_t nj, int64_t ni, int64_t jb, int64_t je, const double* T1, double* T2,
-                   double* residual, cudaStream_t s) {
-  return heat_launch(nj, ni, jb, je, T1, T2, residual, s);
+                   double* residual, cudaStream_t s, const double* res_init) {
+  return heat_launch(nj, ni, jb, je, T1, T2, residual, s, res_init);
 }
 
 }  // namespace xr

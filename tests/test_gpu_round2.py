@@ -185,3 +185,39 @@ def test_colsmall_kernel(op, dtype):
         check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
         init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 5)
         check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
+
+
+@pytest.mark.parametrize("xform,dtype", [("disk", "fp32"), ("disk", "fp64"), ("dot", "int32"), ("dot", "int64"),
+                                         ("dot", "fp32"), ("dot", "fp64")])
+def test_transform_reduce_bulk_ring(xform, dtype):
+    """Whole-array transform-reduce on >= 16 MiB inputs: the two-input bulk
+    ring (xform_stream_kernel).  Disk counts and integer dots are bit-exact
+    against the oracle, fp dots within C9; a ragged tail (n % VEC != 0), init,
+    and a misaligned pair that falls back to the register path."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    npd = oracle.NP_DTYPES[dtype]
+    n = (16 << 20) // np.dtype(npd).itemsize + 3
+    if dtype.startswith("fp"):
+        x = datagen.uniform_float(61, n + 1, -1.0, 1.0, npd)
+        y = datagen.uniform_float(62, n + 1, -1.0, 1.0, npd)
+    else:
+        x = datagen.uniform_int(61, n + 1, -1000, 1000, npd)
+        y = datagen.uniform_int(62, n + 1, -1000, 1000, npd)
+    xd, yd = torch.from_numpy(x).cuda(), torch.from_numpy(y).cuda()
+    odt = torch.int64 if xform == "disk" else torch_dt(dtype)
+    for off in (0, 1):  # 16-B aligned (bulk ring) and misaligned (register path)
+        for init in (None, 7):
+            out = torch.full((1,), 0 if init is None else init, dtype=odt, device="cuda")
+            mask = xr.mask_of("gwv") | (xr.INIT_FROM_OUT if init is not None else 0)
+            assert xr.xr_transform_reduce(xform, dtype, (n, 1, 1), mask, xd[off:].data_ptr(), yd[off:].data_ptr(),
+                                          out.data_ptr(), torch.cuda.current_stream().cuda_stream) == 0
+            ini = None if init is None else np.array([init], dtype=np.int64 if xform == "disk" else npd)
+            ref, S = oracle.transform_reduce(xform, dtype, (n, 1, 1), "gwv", x[off:off + n], y[off:off + n],
+                                             init=ini, want_abs=True)
+            got = out.cpu().numpy()
+            if xform == "disk" or not dtype.startswith("fp"):
+                assert np.array_equal(got, ref), (xform, dtype, off, init, got, ref)
+            else:
+                tau = 1e-5 if dtype == "fp32" else 1e-12
+                assert abs(float(got[0]) - float(ref[0])) <= tau * S[0], (got, ref, S)
