@@ -265,7 +265,7 @@ def run_reference(args):
                          "sample": f"first {sample_n} elements of the workload per step (plain C oracle, 1 thread)"},
         "e2e": {"value": value, "unit": "elements/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
@@ -532,7 +532,7 @@ def run_gpu(args):
         }
         if multi is not None:
             line["multi_gpu"] = multi
-        print(json.dumps(line), flush=True)
+        emit(line)
     if comm is not None:
         comm.close()
     if use_comm:
@@ -540,11 +540,31 @@ def run_gpu(args):
     return 0
 
 
+_JSON_FD = None
+
+
+def emit(line: dict):
+    """The ONE JSON line, on the process's original stdout.  Everything else
+    (NCCL's "NCCL version ..." banner, library prints) was redirected to
+    stderr in main(), so the line stays alone on stdout."""
+    data = (json.dumps(line) + "\n").encode()
+    if _JSON_FD is None:
+        sys.stdout.write(data.decode())
+        sys.stdout.flush()
+    else:
+        os.write(_JSON_FD, data)
+
+
 def main():
+    global _JSON_FD
     args = parse()
     rc = launch_ranks(args)
     if rc is not None:
         return rc
+    # keep stdout for the JSON line only: fd 1 -> stderr for the rest of the run
+    sys.stdout.flush()
+    _JSON_FD = os.dup(1)
+    os.dup2(2, 1)
     if args.impl == "reference":
         return run_reference(args)
     return run_gpu(args)

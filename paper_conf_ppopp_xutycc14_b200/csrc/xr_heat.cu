@@ -371,20 +371,29 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
     const int64_t nrows = j1 - j0 + 2;
     const int64_t qb = q;  // global index of row 0 of this tile
     mbar_wait(&full[(qb + 1) % kHeatSlots], (unsigned)(((qb + 1) / kHeatSlots) & 1));
-    const int64_t col = c0 + 2 * tid;
     const int li = 4 + 2 * tid;
-    const bool i0 = col >= 1 && col <= ni - 2;
-    const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
     const int64_t ws = max(c0 - 2, (int64_t)0);
     constexpr bool odd = ODD;
     for (int64_t r = 1; r < nrows - 1; ++r) {
       const int64_t qd = qb + r + 1;
       mbar_wait(&full[qd % kHeatSlots], (unsigned)((qd / kHeatSlots) & 1));
+      // ODD (ni odd): the rows alternate their 16-B phase.  On a row whose
+      // flat index j*ni + c0 is odd the thread's column pair moves one column
+      // left, so its flat index -- and hence its T2 address and its position
+      // in the row's staged window -- is 16-B aligned: the centre pair loads
+      // and the store are 16-B vectors on every row; only the up / down pairs
+      // (the other phase) are two 8-B loads.  Tile t covers columns
+      // [c0 - p, c0 + 512 - p) on a row of phase p, so every column still
+      // belongs to exactly one tile.
+      const int64_t ecur = (j0 - 1 + r) * ni + ws;  // window start element of the centre row
+      const int p = odd ? (int)(ecur & 1) : 0;      // == phase of (j*ni + c0): ws and c0 are both even
+      const int64_t col = c0 + 2 * tid - p;
+      const bool i0 = col >= 1 && col <= ni - 2;
+      const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
       if (i0 || i1) {
         const double* up = slots[(qb + r - 1) % kHeatSlots];
         const double* cur = slots[(qb + r) % kHeatSlots];
         const double* dn = slots[qd % kHeatSlots];
-        const int64_t ecur = (j0 - 1 + r) * ni + ws;  // window start element of row r
         double2 u2, c2, d2;
         double l, rr;
         if constexpr (!odd) {  // every row 16-B aligned: vector loads
@@ -393,18 +402,20 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
           d2 = *reinterpret_cast<const double2*>(dn + li);
           l = cur[li - 1];
           rr = cur[li + 2];
-        } else {  // rows alternate the staging shift (ni odd)
-          const int su = li + (int)((ecur - ni) & 1), sc = li + (int)(ecur & 1), sd = li + (int)((ecur + ni) & 1);
-          u2 = make_double2(up[su], up[su + 1]);
-          c2 = make_double2(cur[sc], cur[sc + 1]);
-          d2 = make_double2(dn[sd], dn[sd + 1]);
-          l = cur[sc - 1];
-          rr = cur[sc + 2];
+        } else {
+          // centre: column c sits at c - c0 + 4 + p, i.e. li for the pair
+          // (aligned); up / down rows have the other phase 1 - p: li + 1 - 2p
+          const int so = li + 1 - 2 * p;
+          c2 = *reinterpret_cast<const double2*>(cur + li);
+          u2 = make_double2(up[so], up[so + 1]);
+          d2 = make_double2(dn[so], dn[so + 1]);
+          l = cur[li - 1];
+          rr = cur[li + 2];
         }
         const double n0 = stencil(u2.x, d2.x, l, c2.y);
         const double n1 = stencil(u2.y, d2.y, c2.x, rr);
         double* dst = a.T2 + (j0 + r - 1) * ni + col;
-        if (i0 && i1 && !(odd && (((uintptr_t)dst) & 15u))) {
+        if (i0 && i1) {
           __stcs(reinterpret_cast<double2*>(dst), make_double2(n0, n1));
         } else {
           if (i0) __stcs(dst, n0);
