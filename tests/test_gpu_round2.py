@@ -221,3 +221,38 @@ def test_transform_reduce_bulk_ring(xform, dtype):
             else:
                 tau = 1e-5 if dtype == "fp32" else 1e-12
                 assert abs(float(got[0]) - float(ref[0])) <= tau * S[0], (got, ref, S)
+
+
+def test_multi_variable_bulk_ring():
+    """Eight whole-array variables of mixed (op, dtype) on a large nest: the
+    multi-variable bulk ring (one launch); every output against the oracle
+    (integer / bitwise / logical / min / max bit-exact, fp + and * within
+    C9 / C10), with init on half of them, a ragged length, and the same call
+    with one misaligned input (the register path)."""
+    import torch
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    n = (1 << 22) + 5
+    vars_ = [("+", "int32"), ("+", "fp64"), ("max", "fp32"), ("^", "int64"), ("&&", "fp32"), ("*", "int32"),
+             ("min", "int64"), ("+", "fp32")]
+    for off in (0, 1):
+        xs, ds, outs, inits, spec = [], [], [], [], []
+        for k, (op, dt) in enumerate(vars_):
+            x = recipes.make(KIND[op], (n + 1, 1, 1), 7, dt, 300 + k)
+            xd = torch.from_numpy(x).cuda()
+            init = recipes.make("ints", (1, 1, 1), 1, dt, 9 + k) if k % 2 == 0 else None
+            o = torch.zeros(1, dtype=torch_dt(dt), device="cuda")
+            if init is not None:
+                o.copy_(torch.from_numpy(init))
+            src = xd[off:off + n] if k == 3 else xd[:n]  # one misaligned input when off == 1
+            xs.append(x[off:off + n] if k == 3 else x[:n])
+            ds.append(xd)
+            outs.append(o)
+            inits.append(init)
+            spec.append((op, dt, "gwv" if init is None else xr.mask_of("gwv") | xr.INIT_FROM_OUT,
+                         src.data_ptr(), o.data_ptr()))
+        n0 = xr.xr_launch_count()
+        assert xr.xr_reduce_multi_at(spec, (n, 1, 1), torch.cuda.current_stream().cuda_stream) == 0
+        torch.cuda.synchronize()
+        assert xr.xr_launch_count() - n0 == 1
+        for k, (op, dt) in enumerate(vars_):
+            check(op, dt, (n, 1, 1), "gwv", outs[k].cpu().numpy(), xs[k], init=inits[k])
