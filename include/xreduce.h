@@ -242,7 +242,8 @@ typedef struct {
                            7 rows (bulk-streamed short contiguous rows),
                            8 colflat (narrow-row column reduction),
                            9 rkr (bulk-streamed j-blocks of short rows, k loop),
-                           10 colsmall (warp per 32 B of columns, small inputs) */
+                           10 colsmall (warp per 32 B of columns, small inputs),
+                           11 rcluster (one 16-CTA cluster, DSMEM gang tier) */
   int64_t cdims[3];     /* canonical extents (shape-dependent, rest 0)       */
   int64_t out_count;
   int group;            /* seg: lanes per group (8, 32 or the CTA size)      */

@@ -145,6 +145,8 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   Plan p;
   make_plan(op, dtype, dims, mask & 7u, (uint64_t)(uintptr_t)in, sms, &p);
   if (p.kernel == K_NONE) return XR_OK;
+  if (exch && p.kernel == K_RCLUSTER)  // the fused exchange needs a CTA-wide last-CTA tier: seg plan
+    make_plan(op, dtype, dims, mask & 7u, (uint64_t)(uintptr_t)in, sms, &p, /*seg_only=*/true);
   if (exch) {
     const bool ok = p.out_count == 1 &&
                     (p.kernel == K_STREAM || (p.kernel == K_SEG && p.group == kBlock));

@@ -1177,6 +1177,64 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   }
 }
 
+// ------------------------------------------------------------- small whole-array kernel
+// R shape on SMALL inputs (latency bound; e.g. the paper-style testsuite nest
+// at gang+worker+vector, 2 MiB): ONE thread-block cluster of kClusterCtas
+// CTAs x kClusterBlock threads; CTA r folds the contiguous r-th slice with 8
+// 16-B loads in flight per thread (one load round at 2 MiB), a2 + a3 within
+// the CTA, then the gang tier runs through DISTRIBUTED SHARED MEMORY: after a
+// cluster barrier CTA 0 reads the CTAs' values in rank order and writes the
+// output -- no global partials, no atomic ticket, no fence round trips (the
+// seg kernel's last-CTA ticket chain costs ~2 us of a 4 us call).
+template <int OP, typename T>
+__global__ void __launch_bounds__(kClusterBlock) rcluster_kernel(const __grid_constant__ SegArgs a) {
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / sizeof(T);
+  __shared__ Acc smem[32];
+  __shared__ Acc cta_val;
+  pdl_wait();  // no global access above this line
+  pdl_trigger();
+  const unsigned rank = blockIdx.x, nctas = gridDim.x;  // the grid is ONE cluster
+  const int64_t c0 = split_lo_vec(a.L, nctas, rank, VEC), c1 = split_lo_vec(a.L, nctas, rank + 1, VEC);
+  Acc acc[8][VEC];
+#pragma unroll
+  for (int k = 0; k < 8; ++k)
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[k][q] = O::identity();
+  fold_row<OP, T, kClusterBlock, 8>(static_cast<const T*>(a.in) + c0, c1 - c0, threadIdx.x, acc);
+  Acc v = fold_acc<OP, T, 8, VEC>(acc);
+  v = block_reduce<OP, T, kClusterBlock>(v, smem);
+  if (threadIdx.x == 0) cta_val = v;
+  // cluster barrier (release / acquire): every CTA's value is visible in its
+  // shared memory to the other CTAs of the cluster
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+  if (rank == 0 && threadIdx.x == 0) {
+    Acc w = O::identity();
+    const unsigned local = static_cast<unsigned>(__cvta_generic_to_shared(&cta_val));
+#pragma unroll 1
+    for (unsigned r = 0; r < nctas; ++r) {  // rank order: deterministic
+      unsigned remote;
+      asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local), "r"(r));
+      Acc x;
+      if constexpr (sizeof(Acc) == 4) {
+        unsigned b;
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(b) : "r"(remote) : "memory");
+        memcpy(&x, &b, 4);
+      } else {
+        unsigned long long b;
+        asm volatile("ld.shared::cluster.u64 %0, [%1];" : "=l"(b) : "r"(remote) : "memory");
+        memcpy(&x, &b, 8);
+      }
+      w = O::combine(w, x);
+    }
+    T* out = static_cast<T*>(a.out);
+    out[0] = merge_init<OP, T>(w, out, 0, a.init_from_out);
+  }
+  // keep every CTA's shared memory alive until CTA 0 has read it
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
 // ------------------------------------------------------------- small column kernel
 // RK / KRK on SMALL inputs (latency bound, e.g. the paper-style testsuite nest
 // 64 x 64 x 128 at gang or worker level) with few reduced rows (R <= 256):
@@ -1689,6 +1747,43 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
       if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.seg)) return e;
+      break;
+    }
+    case K_RCLUSTER: {
+      // one cluster of 16 CTAs (non-portable size; 8 if the device cannot
+      // co-schedule 16), cluster dimension set at launch
+      auto kern = rcluster_kernel<OP, T>;
+      static int csize[kMaxDevices];  // 0 = not yet probed on that device
+      int dev = 0;
+      if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) { cudaGetLastError(); dev = 0; }
+      int n = __atomic_load_n(&csize[dev], __ATOMIC_RELAXED);
+      cudaLaunchConfig_t cfg = {};
+      cfg.blockDim = dim3(kClusterBlock);
+      cfg.stream = s;
+      cudaLaunchAttribute attr[2];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+      attr[1].id = cudaLaunchAttributeClusterDimension;
+      cfg.attrs = attr;
+      cfg.numAttrs = 2;
+      if (n == 0) {
+        n = 8;
+        if (cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) == cudaSuccess) {
+          int active = 0;
+          cfg.gridDim = dim3(kClusterCtas);
+          attr[1].val.clusterDim.x = kClusterCtas;
+          attr[1].val.clusterDim.y = 1;
+          attr[1].val.clusterDim.z = 1;
+          if (cudaOccupancyMaxActiveClusters(&active, kern, &cfg) == cudaSuccess && active > 0) n = kClusterCtas;
+        }
+        cudaGetLastError();
+        __atomic_store_n(&csize[dev], n, __ATOMIC_RELAXED);
+      }
+      cfg.gridDim = dim3((unsigned)n);
+      attr[1].val.clusterDim.x = (unsigned)n;
+      attr[1].val.clusterDim.y = 1;
+      attr[1].val.clusterDim.z = 1;
+      if (cudaError_t e = cudaLaunchKernelEx(&cfg, kern, p.seg)) return e;
       break;
     }
     case K_COLSMALL: {

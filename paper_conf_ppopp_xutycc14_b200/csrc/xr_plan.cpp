@@ -329,6 +329,26 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     s.Sr = 1; s.Sc = units; s.units = units;
     return;
   }
+  // small whole-array reductions: one thread-block cluster, gang tier through
+  // distributed shared memory (rcluster_kernel) -- 256 KiB to 4 MiB.  OPT-IN
+  // (XR_CLUSTER=1): measured SLOWER than the seg kernel's last-CTA ticket on
+  // the 2 MiB testsuite nest (CUDA-graph replay 5.5 vs 4.0 us, r02h) -- 16
+  // SMs cannot pull 2 MiB from L2 as fast as 128 CTAs on 128 SMs.
+  if (!seg_only && nr == 1 && row_bytes >= (int64_t(256) << 10) && row_bytes <= (int64_t(4) << 20) &&
+      env.get("XR_CLUSTER") != nullptr) {
+    p->kernel = K_RCLUSTER;
+    p->shape = XR_SHAPE_R;
+    p->group = kClusterBlock;
+    p->block = kClusterBlock;
+    p->vec = vec;
+    p->splits = kClusterCtas;
+    p->units = kClusterCtas;
+    p->grid_hint = kClusterCtas;
+    SegArgs& s = p->seg;
+    s.O = 1; s.C = 1; s.L = L; s.rowStride = 0; s.oStride = 0;
+    s.Sr = 1; s.Sc = kClusterCtas; s.units = kClusterCtas;
+    return;
+  }
   int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };

@@ -256,3 +256,27 @@ def test_multi_variable_bulk_ring():
         assert xr.xr_launch_count() - n0 == 1
         for k, (op, dt) in enumerate(vars_):
             check(op, dt, (n, 1, 1), "gwv", outs[k].cpu().numpy(), xs[k], init=inits[k])
+
+
+@pytest.mark.parametrize("op,dtype", [("+", "int32"), ("+", "fp32"), ("*", "fp64"), ("max", "fp32"), ("^", "int64"),
+                                      ("&&", "int32"), ("min", "fp64"), ("||", "fp32")])
+def test_rcluster_kernel(op, dtype, monkeypatch):
+    """Small whole-array reductions (256 KiB - 4 MiB) on the opt-in cluster
+    kernel (XR_CLUSTER=1): one thread-block cluster, gang tier through
+    distributed shared memory (rank order, no ticket).  Ragged lengths, a
+    misaligned start (scalar head), init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_CLUSTER", "1")
+    size = np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for nbytes in (256 << 10, (2 << 20) + 3 * size, 4 << 20):
+        n = nbytes // size
+        dims = (n, 1, 1)
+        assert xr.xr_plan_describe(op, dtype, dims, "gwv", 256)["kernel"] == "rcluster"
+        x = recipes.make(KIND[op], dims, 7, dtype, n % 1000)
+        for offset in (0, 1):
+            check(op, dtype, dims, "gwv", gpu_reduce(op, dtype, dims, "gwv", x, offset=offset), x)
+        init = recipes.make("ints", (1, 1, 1), 1, dtype, 2)
+        check(op, dtype, dims, "gwv", gpu_reduce(op, dtype, dims, "gwv", x, init=init), x, init=init)
+    # the paper-style testsuite nest at gang+worker+vector (P1 closed form)
+    lin = np.arange(64 * 64 * 128, dtype=np.int64).astype(np.int32)
+    assert gpu_reduce("+", "int32", (64, 64, 128), "gwv", lin)[0] == -262144
