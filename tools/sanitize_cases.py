@@ -26,6 +26,8 @@ cases = [
     ("min", "fp32", (999, 1, 33), "g"),           # col (unaligned)
     ("|", "int32", (20, 300, 64), "w"),           # col KRK
     ("+", "int32", (3, 1, 5), "w"),               # ident
+    ("+", "int32", (64, 64, 128), "g"),           # colsmall (r02)
+    ("max", "fp64", (40, 33, 100), "w"),          # colsmall KRK, half-width last group
 ]
 for op, dtype, dims, lv in cases:
     x = recipes.make({"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "^": "bxor", "&&": "land",
@@ -56,4 +58,22 @@ pz = torch.zeros(64 * 32, device="cuda")
 assert xr.xr_reduce_paper("+", "fp32", (8, 8, 1000), "w", xs.data_ptr(), pz.data_ptr(), 16, 8, 128) == 0
 assert xr.xr_reduce_paper("+", "fp32", (8, 8, 1000), "gwv", xs.data_ptr(), pz.data_ptr(), 16, 8, 128) == 0
 torch.cuda.synchronize()
+# round 2: the cluster kernel (opt-in), the two-input and multi-variable rings
+os.environ["XR_CLUSTER"] = "1"
+x = recipes.make("ints", (1 << 17, 1, 1), 7, "int32", 3)
+check("+", "int32", (1 << 17, 1, 1), "gwv", gpu_reduce("+", "int32", (1 << 17, 1, 1), "gwv", x), x)
+del os.environ["XR_CLUSTER"]
+n = 1 << 22  # 16 MiB per fp32 input: xform_stream_kernel
+bx = torch.rand(n, device="cuda") * 2 - 1
+by = torch.rand(n, device="cuda") * 2 - 1
+assert xr.xr_transform_reduce("disk", "fp32", (n, 1, 1), "gwv", bx.data_ptr(), by.data_ptr(), cnt.data_ptr()) == 0
+torch.cuda.synchronize()
+assert int(cnt.item()) == int(oracle.transform_reduce("disk", "fp32", (n, 1, 1), "gwv", bx.cpu().numpy(),
+                                                      by.cpu().numpy())[0])
+mo = [torch.zeros(1, device="cuda") for _ in range(2)] + [torch.zeros(1, dtype=torch.int64, device="cuda")]
+mi = torch.arange(n, dtype=torch.int64, device="cuda")
+assert xr.xr_reduce_multi([("+", "fp32", bx.data_ptr(), mo[0].data_ptr()), ("max", "fp32", by.data_ptr(), mo[1].data_ptr()),
+                           ("+", "int64", mi.data_ptr(), mo[2].data_ptr())], (n, 1, 1), "gwv") == 0  # multi_stream_kernel
+torch.cuda.synchronize()
+assert int(mo[2].item()) == n * (n - 1) // 2
 print("sanitize cases OK")
