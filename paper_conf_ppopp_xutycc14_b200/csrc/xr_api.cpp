@@ -465,7 +465,8 @@ int xr_plan_describe(int op, int dtype, const int64_t nest_dims[3], unsigned lev
   info->units = p.units;
   info->block = p.block;
   int64_t ctas = p.units;
-  if (p.kernel == K_STREAM || p.kernel == K_COLTMA || p.kernel == K_ROWS || p.kernel == K_RKR) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
+  if (p.kernel == K_COLTMA || p.kernel == K_ROWS || p.kernel == K_RKR) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 3);
+  if (p.kernel == K_STREAM) ctas = std::min<int64_t>(p.units, (int64_t)num_sms * 2);  // 2 resident per SM
   if (p.kernel == K_SEG && p.group < p.block) ctas = (p.units + p.block / p.group - 1) / (p.block / p.group);
   if (p.kernel == K_FILL || p.kernel == K_IDENT) ctas = (p.units + kBlock - 1) / kBlock;
   if (p.kernel == K_COLSMALL) ctas = (p.units + kBlock / 32 - 1) / (kBlock / 32);

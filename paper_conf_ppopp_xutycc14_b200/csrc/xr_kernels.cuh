@@ -1444,6 +1444,14 @@ __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_co
 // the worker tier folds the row phases per column in shared memory; the gang
 // tier is the per-tile ticket of col_kernel.  OOB rows/columns of a box are
 // skipped by the consumers, so the fill value never matters.
+// Deferred group tickets: consumer thread 0 resolves a unit's group ticket at
+// the end of the NEXT unit, so the consumers do not wait for the fence +
+// atomic round trip.  MEASURED SLOWER (r02 same-box A/B: 512^3 32-bit G 86.5
+// vs 84.5 us, GW 93.3 vs 90.6 us; the delayed group folds lengthen the end of
+// the launch), so the ticket is resolved at once by default.
+#ifndef XR_COLTMA_DEFER
+#define XR_COLTMA_DEFER 0
+#endif
 template <int OP, typename T, int NS>
 __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
   using O = Op<OP, T>;
@@ -1522,6 +1530,87 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
   const int tid = tid0 - 32, grp = tid % G, ph = tid / G;
   int seq = 0;
   int64_t g = 0;
+  // fold rows [0, n) of a [n][TW] partial block into column tid (< TW):
+  // 16-B L2 loads, NPA row phases x (TW/AV) column groups, 4 rows in flight
+  auto fold_rows = [&](const Acc* base, int64_t n) -> Acc {
+    const int cg = tid % (TW / AV), q2 = tid / (TW / AV);
+    Acc w[AV];
+#pragma unroll
+    for (int q = 0; q < AV; ++q) w[q] = O::identity();
+    int64_t r = q2;
+    for (; r + 3 * NPA < n; r += 4 * NPA) {
+      uint4 y[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) y[k] = __ldcg(reinterpret_cast<const uint4*>(base + (r + k * NPA) * TW + cg * AV));
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+#pragma unroll
+        for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y[k])[q]);
+    }
+    for (; r < n; r += NPA) {
+      const uint4 y = __ldcg(reinterpret_cast<const uint4*>(base + r * TW + cg * AV));
+#pragma unroll
+      for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y)[q]);
+    }
+#pragma unroll
+    for (int q = 0; q < AV; ++q) red[q2][cg * AV + q] = w[q];
+    cons_sync();
+    Acc z = O::identity();
+    if (tid < TW) {
+#pragma unroll
+      for (int p2 = 0; p2 < NPA; ++p2) z = O::combine(z, red[p2][tid]);
+    }
+    return z;
+  };
+  // a4, two levels: unit partial -> group of kGroupFold (its last unit folds
+  // the group in unit order) -> tile (the last group folds the G2 group
+  // partials).  The group ticket of a unit is DEFERRED: consumer thread 0
+  // issues the fence + atomic after the unit's partial store and the
+  // consumers go straight on to the next unit; the returned ticket is read
+  // (and, if this unit was its group's last, the group folded) at the end of
+  // the next unit or after the loop.  The consumers no longer wait for the
+  // fence + atomic round trip of every unit (r01: each unit stalled all 8
+  // consumer warps ~1 us; more, shorter units were then a net loss).
+  unsigned pend_tk = 0u;   // consumer thread 0: ticket value of the pending unit
+  long long pend_u = -1;   // the pending unit (uniform across consumers)
+  auto finish_pending = [&]() {
+    if (pend_u < 0) return;
+    const int64_t b = pend_u / per_b, rem = pend_u - b * per_b;
+    const int64_t tile = rem / a.S, s = rem - tile * a.S;
+    const int64_t tid_tile = b * a.tiles + tile;
+    const int64_t grp_i = s / kGroupFold;
+    const int64_t g0 = grp_i * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
+    if (tid == 0) s_last = (pend_tk == (unsigned)(gsz - 1));
+    cons_sync();
+    pend_u = -1;
+    if (!s_last) return;  // uniform
+    Acc* P1 = partials + tid_tile * a.S * TW;                                  // [S][TW]
+    Acc* P2 = partials + a.B * a.tiles * a.S * TW + tid_tile * a.G2 * TW;      // [G2][TW]
+    unsigned* gt = a.tickets + tid_tile * a.G2;                                // group tickets
+    unsigned* tt = a.tickets + a.B * a.tiles * a.G2 + tid_tile;                // tile ticket
+    const int64_t oc = tile * TW + tid;
+    __threadfence();
+    const Acc w = fold_rows(P1 + g0 * TW, gsz);
+    if (tid == 0) gt[grp_i] = 0u;
+    if (a.G2 == 1) {
+      if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(w, out, b * a.K + oc, a.init_from_out);
+    } else {
+      if (tid < TW) P2[grp_i * TW + tid] = w;
+      cons_sync();
+      if (tid == 0) {
+        const unsigned tk = ticket_add(tt);
+        s_last = (tk == (unsigned)(a.G2 - 1));
+      }
+      cons_sync();
+      if (s_last) {
+        __threadfence();
+        const Acc z = fold_rows(P2, a.G2);
+        if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(z, out, b * a.K + oc, a.init_from_out);
+        if (tid == 0) *tt = 0u;
+      }
+    }
+    cons_sync();  // red is reused
+  };
   while (true) {
     mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
@@ -1577,81 +1666,22 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     }
     if (a.S == 1) {
       if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(v, out, b * a.K + oc, a.init_from_out);
+      cons_sync();  // red is reused by the next unit
     } else {
-      // a4, two levels: unit partial -> group of kGroupFold (its last CTA folds
-      // the group in unit order) -> tile (the last group folds the G2 group partials)
       const int64_t tid_tile = b * a.tiles + tile;
-      Acc* P1 = partials + tid_tile * a.S * TW;                                  // [S][TW]
-      Acc* P2 = partials + a.B * a.tiles * a.S * TW + tid_tile * a.G2 * TW;      // [G2][TW]
-      unsigned* gt = a.tickets + tid_tile * a.G2;                                // group tickets
-      unsigned* tt = a.tickets + a.B * a.tiles * a.G2 + tid_tile;                // tile ticket
-      const int64_t grp_i = s / kGroupFold;
-      const int64_t g0 = grp_i * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
-      // fold rows [0, n) of a [n][TW] partial block into column tid (< TW):
-      // 16-B L2 loads, NPA row phases x (TW/AV) column groups, 4 rows in flight
-      auto fold_rows = [&](const Acc* base, int64_t n) -> Acc {
-        const int cg = tid % (TW / AV), q2 = tid / (TW / AV);
-        Acc w[AV];
-#pragma unroll
-        for (int q = 0; q < AV; ++q) w[q] = O::identity();
-        int64_t r = q2;
-        for (; r + 3 * NPA < n; r += 4 * NPA) {
-          uint4 y[4];
-#pragma unroll
-          for (int k = 0; k < 4; ++k) y[k] = __ldcg(reinterpret_cast<const uint4*>(base + (r + k * NPA) * TW + cg * AV));
-#pragma unroll
-          for (int k = 0; k < 4; ++k)
-#pragma unroll
-            for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y[k])[q]);
-        }
-        for (; r < n; r += NPA) {
-          const uint4 y = __ldcg(reinterpret_cast<const uint4*>(base + r * TW + cg * AV));
-#pragma unroll
-          for (int q = 0; q < AV; ++q) w[q] = O::combine(w[q], reinterpret_cast<const Acc*>(&y)[q]);
-        }
-#pragma unroll
-        for (int q = 0; q < AV; ++q) red[q2][cg * AV + q] = w[q];
-        cons_sync();
-        Acc z = O::identity();
-        if (tid < TW) {
-#pragma unroll
-          for (int p2 = 0; p2 < NPA; ++p2) z = O::combine(z, red[p2][tid]);
-        }
-        return z;
-      };
+      Acc* P1 = partials + tid_tile * a.S * TW;  // [S][TW]
       if (tid < TW) P1[s * TW + tid] = v;
-      cons_sync();  // partial stores happen-before thread 0's (cumulative) fence
-      if (tid == 0) {
-        const unsigned tk = ticket_add(&gt[grp_i]);
-        s_last = (tk == (unsigned)(gsz - 1));
-      }
-      cons_sync();
-      if (s_last) {
-        __threadfence();
-        const Acc w = fold_rows(P1 + g0 * TW, gsz);
-        if (tid == 0) gt[grp_i] = 0u;
-        if (a.G2 == 1) {
-          if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(w, out, b * a.K + oc, a.init_from_out);
-        } else {
-          if (tid < TW) P2[grp_i * TW + tid] = w;
-          cons_sync();
-          if (tid == 0) {
-            const unsigned tk = ticket_add(tt);
-            s_last = (tk == (unsigned)(a.G2 - 1));
-          }
-          cons_sync();
-          if (s_last) {
-            __threadfence();
-            const Acc z = fold_rows(P2, a.G2);
-            if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(z, out, b * a.K + oc, a.init_from_out);
-            if (tid == 0) *tt = 0u;
-          }
-        }
-      }
+      cons_sync();  // partial stores happen-before thread 0's (cumulative) fence; red free
+      finish_pending();  // the previous unit's group (its ticket has long returned)
+      if (tid == 0) pend_tk = ticket_add(&a.tickets[tid_tile * a.G2 + s / kGroupFold]);  // result read later
+      pend_u = u;
+#if !XR_COLTMA_DEFER
+      finish_pending();  // A/B: resolve the ticket right away (the r01 behaviour)
+#endif
     }
-    cons_sync();
     ++seq;
   }
+  finish_pending();
 }
 
 // ------------------------------------------------------------- elementwise
@@ -1690,6 +1720,11 @@ __global__ void __launch_bounds__(kBlock) gather_combine_kernel(const T* g, int 
 }
 
 // ------------------------------------------------------------- host launch
+// Ring depth of the stream kernel (16 KiB stages); the planner sizes units
+// for kStages.  XR_STREAM_NS=6 (A/B build): 96 KiB rings, 2 CTAs / SM.
+#ifndef XR_STREAM_NS
+#define XR_STREAM_NS 4
+#endif
 
 template <int OP, typename T>
 cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
@@ -1723,9 +1758,17 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       break;
     }
     case K_STREAM: {
-      auto kern = stream_kernel<OP, T, kStages, kStageBytes>;
-      constexpr int dyn = kStages * kStageBytes;
-      const int occ = occ_dev<stream_kernel<OP, T, kStages, kStageBytes>>(kWsEpiBlock, dyn);
+      auto kern = stream_kernel<OP, T, XR_STREAM_NS, kStageBytes>;
+      constexpr int dyn = XR_STREAM_NS * kStageBytes;
+      int occ = occ_dev<stream_kernel<OP, T, XR_STREAM_NS, kStageBytes>>(kWsEpiBlock, dyn);
+      // 2 resident CTAs per SM (r02 same-box A/B vs 3: 2^30 fp32 584.2 vs
+      // 588.1 us, 32768^2 rows 578.5 vs 582.0, 512^3 64-bit GV 156.2 vs 158.2,
+      // 32-bit WV 82.5 vs 84.4; 0.5-1 GiB whole arrays equal; 64-bit GWV
+      // 160.2 vs 158.2).  XR_STREAM_CTAS_PER_SM overrides.
+      {
+        const char* e = std::getenv("XR_STREAM_CTAS_PER_SM");
+        occ = std::max(1, std::min(occ, e ? std::atoi(e) : 2));
+      }
       if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kWsEpiBlock), dyn, s,
                                      p.seg))
         return e;

@@ -219,7 +219,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       p->vec = vec;
       p->splits = S;
       p->units = B * tiles * S;
-      p->grid_hint = std::min<int64_t>(cap, cdiv(p->units, std::max<int64_t>(k, cdiv(p->units, cap))));
+      // S == 1 (many column tiles): all resident CTAs claim the tiles
+      // dynamically (r02 grid sweep, 512^3 64-bit G / W: 444 CTAs 158 / 156
+      // us vs 164 / 162 us at the k-units-per-CTA grid of 410); S > 1: k
+      // units per CTA as before
+      p->grid_hint = S == 1 ? std::min<int64_t>(cap, p->units)
+                            : std::min<int64_t>(cap, cdiv(p->units, std::max<int64_t>(k, cdiv(p->units, cap))));
+      if (const char* eg = env.get("XR_COLTMA_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
       p->group = kBlock;
       p->sched = true;
       // two-level gang tier: groups of kGroupFold unit partials, then the groups
@@ -293,7 +299,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     p->splits = S;
     p->units = njb * S;
     p->sched = true;
-    p->grid_hint = std::min<int64_t>(cap, p->units);
+    // 2 CTAs per SM (r02 grid sweep, 512^3 32-bit GV: 88.5 us at 222 / 296
+    // CTAs vs 90.4-91.5 us at 444)
+    p->grid_hint = std::min<int64_t>((int64_t)std::max(num_sms, 1) * 2, p->units);
+    if (const char* eg = env.get("XR_RKR_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
     if (S > 1) {
       p->ws_bytes = O * S * asz;
       p->tickets = O;
@@ -324,6 +333,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     p->units = units;
     p->sched = true;
     p->grid_hint = std::min<int64_t>(cap, cdiv(units, k));
+    if (const char* eg = env.get("XR_ROWS_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
     SegArgs& s = p->seg;
     s.O = O; s.C = 1; s.L = L; s.rowStride = 0; s.oStride = L;
     s.Sr = 1; s.Sc = units; s.units = units;
