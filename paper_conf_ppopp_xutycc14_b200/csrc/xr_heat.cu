@@ -511,7 +511,9 @@ static int heat_launch(int64_t nj, int64_t ni, int64_t jb, int64_t je, const dou
     pa.gx = gx;
     pa.gy = gy;
     pa.sched = reinterpret_cast<unsigned long long*>(tickets + 2);  // after the residual ticket (8-B aligned)
-    const int64_t pgrid = std::min<int64_t>(gx * gy, (int64_t)sms * occ);
+    int occ_use = occ;
+    if (const char* e = std::getenv("XR_HEAT_CTAS_PER_SM")) occ_use = std::max(1, std::min(occ, std::atoi(e)));  // A/B
+    const int64_t pgrid = std::min<int64_t>(gx * gy, (int64_t)sms * occ_use);
     if (odd) le = launch_pdl(heat_persistent_kernel<true>, dim3((unsigned)pgrid), dim3(kWsBlock), 0, s, pa);
     else le = launch_pdl(heat_persistent_kernel<false>, dim3((unsigned)pgrid), dim3(kWsBlock), 0, s, pa);
   } else if (bulk) le = launch_pdl(heat_bulk_kernel, grid, dim3(kWsBlock), 0, s, a);
