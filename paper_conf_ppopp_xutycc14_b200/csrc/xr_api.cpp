@@ -168,6 +168,7 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   p.seg.tl = debug_timeline();
   p.col.in = in; p.col.out = out; p.col.partials = w.partials; p.col.tickets = w.tickets;
   p.col.init_from_out = ifo;
+  p.col.tl = debug_timeline();
   p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
   p.rkr.in = in; p.rkr.out = out; p.rkr.partials = w.partials; p.rkr.tickets = w.tickets;
   p.rkr.sched = sched; p.rkr.init_from_out = ifo;

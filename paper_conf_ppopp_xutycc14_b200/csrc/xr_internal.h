@@ -65,6 +65,7 @@ struct SegArgs {
   int64_t Sr, Sc;      // splits over rows and over columns; S = Sr*Sc per output
   int64_t units;       // O * S
   int init_from_out;
+  int packed;            // seg kernel, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[O]
   int use_exch;          // 1: fused exchange of the O == 1 result (exch below)
   ExchArgs exch;
   unsigned long long* tl;  // profiling timeline (xr_debug_timeline), null when off
@@ -83,6 +84,7 @@ struct ColArgs {
   int64_t units;       // B * tiles * S
   int64_t G2;          // coltma: groups of kGroupFold unit partials per tile (two-level gang tier)
   int init_from_out;
+  unsigned long long* tl;  // profiling timeline (coltma; xr_debug_timeline), null when off
 };
 
 constexpr int kGroupFold = 64;  // unit partials folded per group by the group's last CTA

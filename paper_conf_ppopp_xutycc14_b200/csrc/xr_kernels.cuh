@@ -299,6 +299,14 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
           if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
           else out[o] = r;
         }
+      } else if (PackedAdd<OP, T>::value && a.packed) {  // a4 in one atomic (32-bit int '+')
+        uint32_t sum;
+        if (threadIdx.x == 0 &&
+            packed_add_arrive(reinterpret_cast<unsigned long long*>(a.tickets) + o, (uint32_t)v, S, &sum)) {
+          const T r = merge_init<OP, T>((Acc)sum, out, o, a.init_from_out);
+          if (a.use_exch) peer_exchange<OP, T>(a.exch, out, r);
+          else out[o] = r;
+        }
       } else {  // a4: gang tier, last CTA of output o combines its S partials
         if (threadIdx.x == 0) {
           partials[u] = v;
@@ -338,6 +346,11 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
       v = group_reduce<OP, T, W>(v);
       if (S == 1) {
         if (active && lane == 0) out[o] = merge_init<OP, T>(v, out, o, a.init_from_out);
+      } else if (PackedAdd<OP, T>::value && a.packed) {  // a4 in one atomic (32-bit int '+')
+        uint32_t sum;
+        if (active && lane == 0 &&
+            packed_add_arrive(reinterpret_cast<unsigned long long*>(a.tickets) + o, (uint32_t)v, S, &sum))
+          out[o] = merge_init<OP, T>((Acc)sum, out, o, a.init_from_out);
       } else {  // W == 32 here: the warp is one group, `active` is warp-uniform
         int last = 0;
         if (lane == 0) {
@@ -1494,10 +1507,12 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
   if (warp == 0) {
     // ---------------- producer warp
     if (lane == 0) {
+      tl_event(a.tl, TL_START, 0);
       int64_t g = 0;
       int seq = 0;
       long long u = claim_first(a.sched);
       while (true) {
+        tl_event(a.tl, TL_UNIT, u);
         const long long nu = claim_next(a.sched);
         const int slot0 = (int)(g % NS);
         s_units[seq & (RING - 1)] = u < a.units ? u : -1;
@@ -1664,6 +1679,7 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
 #pragma unroll
       for (int p2 = 0; p2 < NPH; ++p2) v = O::combine(v, red[p2][tid]);
     }
+    if (tid == 0) tl_event(a.tl, TL_UNIT_DONE, u);
     if (a.S == 1) {
       if (tid < TW && oc < a.K) out[b * a.K + oc] = merge_init<OP, T>(v, out, b * a.K + oc, a.init_from_out);
       cons_sync();  // red is reused by the next unit
@@ -1681,7 +1697,9 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     }
     ++seq;
   }
+  if (tid == 0) tl_event(a.tl, TL_CONS_END, 0);
   finish_pending();
+  if (tid == 0) tl_event(a.tl, TL_END, 0);
 }
 
 // ------------------------------------------------------------- elementwise

@@ -227,6 +227,27 @@ namespace xr {
 #ifndef XR_TICKET_ACQREL
 #define XR_TICKET_ACQREL 0
 #endif
+// Packed gang tier for 32-bit integer '+' (exact and order-free mod 2^32):
+// one 64-bit word per output carries the running sum in the high half and the
+// arrival count in the low half, so ONE relaxed atomic both deposits a
+// split's partial and takes its ticket -- no partial store, no fence, no
+// reload of the partials by the last arriver (the sum is in the atomic's
+// return value).  The count never carries into the sum (S < 2^32); the sum's
+// carry out of bit 63 drops, which is the mod-2^32 wrap of the result.
+template <int OP, typename T>
+struct PackedAdd {
+  static constexpr bool value = OP == OP_ADD && !IsFp<T>::value && sizeof(T) == 4;
+};
+// Returns true for the last of S arrivals, with the total in *sum; that
+// arrival resets the word for the next launch.
+__device__ __forceinline__ bool packed_add_arrive(unsigned long long* w, uint32_t v, int64_t S, uint32_t* sum) {
+  const unsigned long long old = atomicAdd(w, ((unsigned long long)v << 32) | 1ull);
+  if ((uint32_t)old != (uint32_t)(S - 1)) return false;
+  *sum = (uint32_t)(old >> 32) + v;
+  *w = 0ull;
+  return true;
+}
+
 __device__ __forceinline__ unsigned ticket_add(unsigned* t) {
 #if XR_TICKET_ACQREL
   unsigned v;

@@ -410,6 +410,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   if (S > 1) {
     p->ws_bytes = O * S * asz;
     p->tickets = O;
+    // seg, 32-bit integer '+': the packed gang tier (xr_ops.cuh PackedAdd)
+    // keeps sum and count of an output in one 64-bit word, no partials
+    if (!stream && !seg_only && op == XR_OP_ADD && dtype == XR_INT32 && env.get("XR_NO_PACKED") == nullptr) {
+      p->ws_bytes = 0;
+      p->tickets = 2 * O;
+      p->seg.packed = 1;
+    }
   }
   if (stream && O == 1) {  // unit partials + one CTA-exit ticket, also when S == 1
     p->ws_bytes = std::max<int64_t>(S, 1) * asz;

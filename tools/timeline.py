@@ -31,18 +31,20 @@ def q(a, ps=(0, 10, 50, 90, 100)):
     return {f"p{p}": round(float(np.percentile(a, p)), 3) for p in ps} if a.size else {}
 
 
-def run(n, dtype, op, reps):
+def run(n, dtype, op, reps, nest=None, mask="gwv"):
     tdt = {"fp32": torch.float32, "int64": torch.int64, "fp64": torch.float64, "int32": torch.int32}[dtype]
+    nest = tuple(nest) if nest else (n, 1, 1)
+    n = int(np.prod(nest))
     x = torch.ones(n, dtype=tdt, device="cuda")
-    out = torch.zeros(1, dtype=tdt, device="cuda")
+    out = torch.zeros(max(1, xr.xr_out_count(nest, mask)), dtype=tdt, device="cuda")
     s = torch.cuda.current_stream()
     for _ in range(3):
-        assert xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), s.cuda_stream) == 0
+        assert xr.xr_reduce(op, dtype, nest, mask, x.data_ptr(), out.data_ptr(), s.cuda_stream) == 0
     torch.cuda.synchronize()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
     for a, b in evs:
         a.record(s)
-        xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), s.cuda_stream)
+        xr.xr_reduce(op, dtype, nest, mask, x.data_ptr(), out.data_ptr(), s.cuda_stream)
         b.record(s)
     torch.cuda.synchronize()
     ms = sorted(a.elapsed_time(b) for a, b in evs)
@@ -56,7 +58,7 @@ def run(n, dtype, op, reps):
         xr._lib.xr_debug_timeline(buf.data_ptr(), cap)
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(s)
-        xr.xr_reduce(op, dtype, (n, 1, 1), "gwv", x.data_ptr(), out.data_ptr(), s.cuda_stream)
+        xr.xr_reduce(op, dtype, nest, mask, x.data_ptr(), out.data_ptr(), s.cuda_stream)
         b.record(s)
         xr._lib.xr_debug_timeline(None, 0)
         torch.cuda.synchronize()
@@ -80,11 +82,11 @@ def run(n, dtype, op, reps):
     for c in np.unique(cta):
         tt = np.sort(us[(cta == c) & (ev == 2)])
         ud += list(np.diff(tt))
-    plan = xr.xr_plan_describe(op, dtype, (n, 1, 1), "gwv", x.data_ptr())
+    plan = xr.xr_plan_describe(op, dtype, nest, mask, x.data_ptr())
     bytes_ = n * x.element_size()
     span = float(end.max()) if end.size else float(cons_end.max())
     return {
-        "elements": n, "dtype": dtype, "bytes": bytes_, "plan": {k: plan[k] for k in ("kernel", "units", "grid")},
+        "elements": n, "nest": list(nest), "mask": mask, "dtype": dtype, "bytes": bytes_, "plan": {k: plan[k] for k in ("kernel", "units", "grid")},
         "event_ms_median": ms[len(ms) // 2], "event_ms_min": ms[0],
         "timeline_event_ms": ev_ms,
         "span_us_first_start_to_out": span,
@@ -97,6 +99,8 @@ def run(n, dtype, op, reps):
         "units_per_cta": q(units_per_cta),
         "unit_us": q(ud),
         "records": int(len(r)),
+        "last_real_claim_us": float(us[(ev == 1) & (unit < int(plan["units"]))].max()),
+        "unit_done_last_us": float(us[ev == 2].max()) if (ev == 2).any() else None,
     }
 
 
@@ -107,10 +111,12 @@ def main():
     ap.add_argument("--op", default="+")
     ap.add_argument("--reps", type=int, default=20)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--nest", type=int, nargs=3, default=None, help="3-level nest (overrides --elements)")
+    ap.add_argument("--mask", default="gwv")
     a = ap.parse_args()
     lines = []
-    for n in a.elements:
-        d = run(n, a.dtype, a.op, a.reps)
+    for n in ([0] if a.nest else a.elements):
+        d = run(n, a.dtype, a.op, a.reps, a.nest, a.mask)
         lines.append(json.dumps(d))
         print(lines[-1], flush=True)
     if a.out:
