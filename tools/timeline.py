@@ -70,6 +70,9 @@ def run(n, dtype, op, reps, nest=None, mask="gwv"):
     ev = ((r[:, 0] >> np.uint64(32)) & np.uint64(0xff)).astype(np.int64)
     unit = (r[:, 0] & np.uint64(0xffffffff)).astype(np.int64)
     t = r[:, 1].astype(np.int64)
+    if not (ev == 0).any():
+        return {"elements": n, "nest": list(nest), "mask": mask, "dtype": dtype,
+                "event_ms_median": ms[len(ms) // 2], "timeline": "none (kernel not instrumented)"}
     t0 = t[ev == 0].min()
     us = (t - t0) / 1e3
     starts = us[ev == 0]
