@@ -172,7 +172,7 @@ static int reduce_device(int op, int dtype, const int64_t* dims, unsigned mask, 
   p.elt.in = in; p.elt.out = out; p.elt.init_from_out = ifo;
   p.rkr.in = in; p.rkr.out = out; p.rkr.partials = w.partials; p.rkr.tickets = w.tickets;
   p.rkr.sched = sched; p.rkr.init_from_out = ifo;
-  if (p.kernel == K_COLTMA && !make_col_tmap(&p.tmap, dtype, in, p.col.B, p.col.R, p.col.K)) {
+  if (p.kernel == K_COLTMA && !make_col_tmap(&p.tmap, dtype, in, p.col.B, p.col.R, p.col.K, p.col.box)) {
     // no tensor-map support (driver entry point or encode failed): re-plan
     // onto the register column kernels and launch those instead
     Plan q;

@@ -316,7 +316,7 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
   pdl_trigger();
   if (warp == 0) {  // ---------------- producer warp
     if (lane == 0) {
-      int64_t q = 0;  // global row counter (slot = q % kHeatSlots)
+      unsigned q = 0;  // global row counter (slot = q % kHeatSlots, phase = q / kHeatSlots)
       int seq = 0;
       long long t = claim_first(pa.sched);
       while (true) {
@@ -325,7 +325,7 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
         s_tiles[seq & (RING - 1)] = t < ntiles ? t : -1;
         ++seq;
         if (t >= ntiles) {
-          if (q >= kHeatSlots) mbar_wait(&empty[slot0], (unsigned)(((q / kHeatSlots) - 1) & 1));
+          if (q >= kHeatSlots) mbar_wait(&empty[slot0], ((q / kHeatSlots) - 1) & 1u);
           mbar_arrive(&full[slot0]);
           break;
         }
@@ -346,7 +346,7 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
             if (e - sh + cnt > total) cnt -= 2;
           }
           const unsigned wbytes = (unsigned)(cnt * 8);
-          if (q >= kHeatSlots) mbar_wait(&empty[slot], (unsigned)(((q / kHeatSlots) - 1) & 1));
+          if (q >= kHeatSlots) mbar_wait(&empty[slot], ((q / kHeatSlots) - 1) & 1u);
           mbar_expect_tx(&full[slot], wbytes);
           bulk_g2s(&slots[slot][soff + 2], a.T1 + e - sh, wbytes, &full[slot]);
         }
@@ -357,42 +357,49 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
     return;
   }
   // ---------------- consumer warps
+  // Ring bookkeeping in 32-bit unsigned counters and per-tile invariants
+  // hoisted out of the row loop: the r01 loop recomputed 64-bit signed
+  // modulo / division / row-address products per row (163 warp instructions
+  // per row, issue slots 85 % busy in ncu r02x -- the sweep was issue bound,
+  // not memory bound).
+  static_assert((kHeatSlots & (kHeatSlots - 1)) == 0, "ring slots: power of two");
   const int tid = tid0 - 32, cw = warp - 1;
   double err = 0.0;
   int seq = 0;
-  int64_t q = 0;  // global row counter, as the producer's
+  unsigned q = 0;  // global row counter, as the producer's
+  const int li = 4 + 2 * tid;
   while (true) {
-    mbar_wait(&full[q % kHeatSlots], (unsigned)((q / kHeatSlots) & 1));  // first row of the tile
+    mbar_wait(&full[q % kHeatSlots], (q / kHeatSlots) & 1u);  // first row of the tile
     const long long t = s_tiles[seq & (RING - 1)];
     ++seq;
     if (t < 0) break;
     int64_t c0, j0, j1;
     tile_geom(t, &c0, &j0, &j1);
-    const int64_t nrows = j1 - j0 + 2;
-    const int64_t qb = q;  // global index of row 0 of this tile
-    mbar_wait(&full[(qb + 1) % kHeatSlots], (unsigned)(((qb + 1) / kHeatSlots) & 1));
-    const int li = 4 + 2 * tid;
-    const int64_t ws = max(c0 - 2, (int64_t)0);
+    const int nout = (int)(j1 - j0);  // output rows j0 .. j1-1 (loaded rows j0-1 .. j1)
+    const unsigned qb = q;            // ring index of row j0-1
+    mbar_wait(&full[(qb + 1) % kHeatSlots], ((qb + 1) / kHeatSlots) & 1u);
     constexpr bool odd = ODD;
-    for (int64_t r = 1; r < nrows - 1; ++r) {
-      const int64_t qd = qb + r + 1;
-      mbar_wait(&full[qd % kHeatSlots], (unsigned)((qd / kHeatSlots) & 1));
-      // ODD (ni odd): the rows alternate their 16-B phase.  On a row whose
-      // flat index j*ni + c0 is odd the thread's column pair moves one column
-      // left, so its flat index -- and hence its T2 address and its position
-      // in the row's staged window -- is 16-B aligned: the centre pair loads
-      // and the store are 16-B vectors on every row; only the up / down pairs
-      // (the other phase) are two 8-B loads.  Tile t covers columns
-      // [c0 - p, c0 + 512 - p) on a row of phase p, so every column still
-      // belongs to exactly one tile.
-      const int64_t ecur = (j0 - 1 + r) * ni + ws;  // window start element of the centre row
-      const int p = odd ? (int)(ecur & 1) : 0;      // == phase of (j*ni + c0): ws and c0 are both even
-      const int64_t col = c0 + 2 * tid - p;
-      const bool i0 = col >= 1 && col <= ni - 2;
-      const bool i1 = col + 1 >= 1 && col + 1 <= ni - 2;
+    // ODD (ni odd): the rows alternate their 16-B phase.  On a row whose
+    // flat index j*ni + c0 is odd the thread's column pair moves one column
+    // left, so its flat index -- and hence its T2 address and its position
+    // in the row's staged window -- is 16-B aligned: the centre pair loads
+    // and the store are 16-B vectors on every row; only the up / down pairs
+    // (the other phase) are two 8-B loads.  Tile t covers columns
+    // [c0 - p, c0 + 512 - p) on a row of phase p, so every column still
+    // belongs to exactly one tile.  The window start ws is even and ni odd,
+    // so the phase of output row j -- the parity of j*ni + ws -- is j & 1.
+    const int64_t colA = c0 + 2 * tid;
+    const bool a0 = colA >= 1 && colA <= ni - 2, a1 = colA + 1 >= 1 && colA + 1 <= ni - 2;  // phase 0
+    const bool b0 = colA - 1 >= 1 && colA - 1 <= ni - 2, b1 = colA >= 1 && colA <= ni - 2;  // phase 1
+    double* dst = a.T2 + j0 * ni + colA;  // output row j0, column pair of phase 0
+    for (int r = 1; r <= nout; ++r, dst += ni) {
+      const unsigned qd = qb + (unsigned)r + 1u;
+      mbar_wait(&full[qd % kHeatSlots], (qd / kHeatSlots) & 1u);
+      const int p = odd ? (int)((j0 + r - 1) & 1) : 0;  // phase of output row j0 + r - 1
+      const bool i0 = p ? b0 : a0, i1 = p ? b1 : a1;
       if (i0 || i1) {
-        const double* up = slots[(qb + r - 1) % kHeatSlots];
-        const double* cur = slots[(qb + r) % kHeatSlots];
+        const double* up = slots[(qb + (unsigned)r - 1u) % kHeatSlots];
+        const double* cur = slots[(qb + (unsigned)r) % kHeatSlots];
         const double* dn = slots[qd % kHeatSlots];
         double2 u2, c2, d2;
         double l, rr;
@@ -414,27 +421,34 @@ __global__ void __launch_bounds__(kWsBlock, ODD ? 4 : 1) heat_persistent_kernel(
         }
         const double n0 = stencil(u2.x, d2.x, l, c2.y);
         const double n1 = stencil(u2.y, d2.y, c2.x, rr);
-        double* dst = a.T2 + (j0 + r - 1) * ni + col;
+        double* d = dst - p;
         if (i0 && i1) {
-          __stcs(reinterpret_cast<double2*>(dst), make_double2(n0, n1));
+          __stcs(reinterpret_cast<double2*>(d), make_double2(n0, n1));
         } else {
-          if (i0) __stcs(dst, n0);
-          if (i1) __stcs(dst + 1, n1);
+          if (i0) __stcs(d, n0);
+          if (i1) __stcs(d + 1, n1);
         }
-        if (i0) err = O::combine(err, fabs(__dadd_rn(c2.x, -n0)));
-        if (i1) err = O::combine(err, fabs(__dadd_rn(c2.y, -n1)));
+        // |T1 - T2| is +0 or positive (or NaN), and err starts at +0: on that
+        // domain the reading-C7 max (Op<OP_MAX>::combine: bit-AND of equal
+        // operands, a NaN operand ignored) IS fmax, without its +-0 handling
+        // (r02ac SASS: 18 instructions per combine -> DSETP/SEL)
+        if (i0) err = fmax(err, fabs(__dadd_rn(c2.x, -n0)));
+        if (i1) err = fmax(err, fabs(__dadd_rn(c2.y, -n1)));
       }
-      fence_proxy_async_smem();  // generic reads before the async refill
+      // Row r-1 is dead: every value loaded from it was consumed above (the
+      // stencil's adds issue only once their shared-memory loads returned),
+      // so the release-arrive on `empty` orders the producer's refill after
+      // those reads without a per-row proxy fence (MEMBAR + FENCE.VIEW.ASYNC,
+      // the loop's top stall in r02ac) -- the pattern of TMA load pipelines.
       __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[(qb + r - 1) % kHeatSlots]);  // row r-1 is dead
+      if (lane == 0) mbar_arrive(&empty[(qb + (unsigned)r - 1u) % kHeatSlots]);
     }
-    fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) {  // the tile's last two rows
-      mbar_arrive(&empty[(qb + nrows - 2) % kHeatSlots]);
-      mbar_arrive(&empty[(qb + nrows - 1) % kHeatSlots]);
+      mbar_arrive(&empty[(qb + (unsigned)nout) % kHeatSlots]);
+      mbar_arrive(&empty[(qb + (unsigned)nout + 1u) % kHeatSlots]);
     }
-    q = qb + nrows;
+    q = qb + (unsigned)nout + 2u;
   }
   err = cons_reduce<OP_MAX, double>(err, smem, cw, lane);
   if (tid == 0) {

@@ -83,6 +83,7 @@ struct ColArgs {
   int64_t tiles, S;
   int64_t units;       // B * tiles * S
   int64_t G2;          // coltma: groups of kGroupFold unit partials per tile (two-level gang tier)
+  int box;             // coltma: TMA box width in bytes (256, 512 or 1024; tile = box columns)
   int init_from_out;
   unsigned long long* tl;  // profiling timeline (coltma; xr_debug_timeline), null when off
 };
@@ -166,7 +167,7 @@ cudaError_t gather_f64(int op, const void* g, int nranks, int64_t n, void* out, 
 // Encode the K_COLTMA tensor map for `in` (false if the driver entry point or
 // the encode fails; the caller then re-plans with no_tma and launches the
 // register column kernel instead).
-bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K);
+bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K, int box_bytes);
 
 // Grid for `units` work items given the device's resident-CTA budget.
 int64_t grid_for(int64_t units, int num_sms, int ctas_per_sm);

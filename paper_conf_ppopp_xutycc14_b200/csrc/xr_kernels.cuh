@@ -1465,14 +1465,14 @@ __global__ void __launch_bounds__(BLOCK, XR_COL_MINB) col_kernel(const __grid_co
 #ifndef XR_COLTMA_DEFER
 #define XR_COLTMA_DEFER 0
 #endif
-template <int OP, typename T, int NS>
+template <int OP, typename T, int NS, int BW>  // BW: box width in bytes (one box row)
 __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __grid_constant__ CUtensorMap tmap, ColArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
   constexpr int BLOCK = kConsThreads;        // consumer threads
   constexpr int VEC = 16 / sizeof(T);
-  constexpr int TW = 1024 / (int)sizeof(T);  // box columns
-  constexpr int BR = kStageBytes / 1024;     // box rows
+  constexpr int TW = BW / (int)sizeof(T);    // box columns
+  constexpr int BR = kStageBytes / BW;       // box rows
   constexpr int G = TW / VEC;                // 16-B column groups per row
   constexpr int NPH = BLOCK / G;             // row phases
   constexpr int RING = 8;
@@ -1649,7 +1649,7 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
       if (col_ok && rbase + BR <= r1) {  // full box: all BR / NPH loads in flight, then fold
         U128 x[BR / NPH];
 #pragma unroll
-        for (int i = 0; i < BR / NPH; ++i) x[i] = *reinterpret_cast<const U128*>(st + (ph + i * NPH) * 1024 + grp * 16);
+        for (int i = 0; i < BR / NPH; ++i) x[i] = *reinterpret_cast<const U128*>(st + (ph + i * NPH) * BW + grp * 16);
 #pragma unroll
         for (int i = 0; i < BR / NPH; ++i)
 #pragma unroll
@@ -1659,7 +1659,7 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
         for (int i = 0; i < BR / NPH; ++i) {
           const int row = ph + i * NPH;
           if (col_ok && rbase + row < r1) {
-            const U128 x = *reinterpret_cast<const U128*>(st + row * 1024 + grp * 16);
+            const U128 x = *reinterpret_cast<const U128*>(st + row * BW + grp * 16);
 #pragma unroll
             for (int q = 0; q < VEC; ++q) acc[i & 1][q] = O::combine(acc[i & 1][q], O::lift(unpack<T>(x, q)));
           }
@@ -1858,12 +1858,17 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       break;
     }
     case K_COLTMA: {
-      auto kern = coltma_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
-      const int occ = occ_dev<coltma_kernel<OP, T, kStages>>(kWsBlock, dyn);
-      int64_t grid = grid_for(p.units, num_sms, occ);
-      if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.tmap, p.col)) return e;
+      auto go = [&](auto kern, int occ) -> cudaError_t {
+        int64_t grid = grid_for(p.units, num_sms, occ);
+        if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
+        return launch_pdl(kern, dim3((unsigned)grid), dim3(kWsBlock), dyn, s, p.tmap, p.col);
+      };
+      cudaError_t e;
+      if (p.col.box == 256) e = go(coltma_kernel<OP, T, kStages, 256>, occ_dev<coltma_kernel<OP, T, kStages, 256>>(kWsBlock, dyn));
+      else if (p.col.box == 512) e = go(coltma_kernel<OP, T, kStages, 512>, occ_dev<coltma_kernel<OP, T, kStages, 512>>(kWsBlock, dyn));
+      else e = go(coltma_kernel<OP, T, kStages, 1024>, occ_dev<coltma_kernel<OP, T, kStages, 1024>>(kWsBlock, dyn));
+      if (e) return e;
       break;
     }
     case K_COL: {

@@ -191,30 +191,48 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
     if (!seg_only && !seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr && !no_tma) {
-      const int64_t TWt = 1024 / size, BR = kStageBytes / 1024;
-      const int64_t tiles = cdiv(K, TWt);
       // Balance (measured r01 sweeps): the producer warp keeps every CTA's ring
       // full, so few long units per CTA are best, but the unit count must be an
       // exact multiple of the CTAs launched (896 units on 444 CTAs left 8
       // stragglers for a third round).  k units per CTA, grid = units / k.
       const int64_t cap = (int64_t)std::max(num_sms, 1) * 3;  // resident CTAs (64 KiB ring each)
-      const int64_t base = B * tiles;
       const char* upc = env.get("XR_COLTMA_UNITS_PER_CTA");  // tuning override
-      // measured (r01 sweeps): 2 units per CTA is best with few column tiles
-      // (512^3 G/W/GW: 0.95/0.95/0.97 at 1 GiB); with many tiles (cfg3: 128)
-      // ~512 KiB units (up to 16 per CTA) win (1.04 vs 1.02)
-      const int64_t k_auto = base >= 64
-          ? std::min<int64_t>(16, std::max<int64_t>(2, (B * R * K * size) / (cap << 19))) : 2;
-      const int64_t k = upc ? std::max(1, std::atoi(upc)) : k_auto;
-      int64_t S;
-      if (base >= k * cap) {
-        S = 1;
-      } else {
-        S = std::max<int64_t>(1, (k * cap) / base);
-        S = std::min<int64_t>(S, std::max<int64_t>(1, R / (kStages * BR)));  // >= kStages boxes per unit
+      int64_t tiles = 0, k = 0, BR = 0, TWt = 0;
+      // box = bx bytes x (16 KiB / bx) rows; a tile is bx bytes of columns
+      auto splits_for = [&](int bx) {
+        TWt = bx / size;
+        BR = kStageBytes / bx;
+        tiles = cdiv(K, TWt);
+        const int64_t base = B * tiles;
+        // measured (r01 sweeps): 2 units per CTA is best with few column tiles
+        // (512^3 G/W/GW: 0.95/0.95/0.97 at 1 GiB); with many tiles (cfg3: 128)
+        // ~512 KiB units (up to 16 per CTA) win (1.04 vs 1.02)
+        const int64_t k_auto = base >= 64
+            ? std::min<int64_t>(16, std::max<int64_t>(2, (B * R * K * size) / (cap << 19))) : 2;
+        k = upc ? std::max(1, std::atoi(upc)) : k_auto;
+        int64_t S;
+        if (base >= k * cap) {
+          S = 1;
+        } else {
+          S = std::max<int64_t>(1, (k * cap) / base);
+          S = std::min<int64_t>(S, std::max<int64_t>(1, R / (kStages * BR)));  // >= kStages boxes per unit
+        }
+        if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * 8));
+        return std::max<int64_t>(1, std::min<int64_t>(S, R));
+      };
+      // Box width (r02ac same-process interleaved A/B, tools/ab_env.py,
+      // profiles/ab_box_r02ac.jsonl): 8-byte split tiles (S > 1, the 64-bit GW
+      // cells) stream best in 256-B boxes (165.1 vs 170.8 us); every other
+      // measured shape is best or level at 1 KiB (64-bit G +1.3-1.5 %,
+      // 32-bit G / W and GW within 1 %, cfg3 columns +0.8-0.9 % with narrower
+      // boxes).
+      int box = (size == 8 && splits_for(1024) > 1) ? 256 : 1024;
+      if (const char* eb = env.get("XR_COLTMA_BOX")) {  // A/B override
+        const int v = std::atoi(eb);
+        if (v == 256 || v == 512 || v == 1024) box = v;
       }
-      if (chain_capped) S = std::max<int64_t>(S, cdiv(R, (int64_t)kChainCap * 8));
-      S = std::max<int64_t>(1, std::min<int64_t>(S, R));
+      if (K * size < box) box = 1024;  // (K * size >= 1024 here)
+      const int64_t S = splits_for(box);
       p->kernel = K_COLTMA;
       p->vec = vec;
       p->splits = S;
@@ -235,7 +253,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
         p->tickets = B * tiles * (G2 + 1);
       }
       ColArgs& c = p->col;
-      c.B = B; c.R = R; c.K = K; c.tiles = tiles; c.S = S; c.units = p->units; c.G2 = G2;
+      c.B = B; c.R = R; c.K = K; c.tiles = tiles; c.S = S; c.units = p->units; c.G2 = G2; c.box = box;
       return;
     }
     const int64_t TW = 32 * cv;

@@ -28,7 +28,7 @@ static PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K) {
+bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t R, int64_t K, int box_bytes) {
   if (std::getenv("XR_TEST_TMAP_FAIL") != nullptr) return false;  // test hook: the re-plan fallback
   auto fn = encode_fn();
   if (!fn) return false;
@@ -42,7 +42,7 @@ bool make_col_tmap(CUtensorMap* m, int dtype, const void* in, int64_t B, int64_t
   }
   const cuuint64_t dims[3] = {(cuuint64_t)K, (cuuint64_t)R, (cuuint64_t)B};
   const cuuint64_t strides[2] = {(cuuint64_t)(K * size), (cuuint64_t)(R * K * size)};
-  const cuuint32_t box[3] = {(cuuint32_t)(1024 / size), (cuuint32_t)(kStageBytes / 1024), 1u};
+  const cuuint32_t box[3] = {(cuuint32_t)(box_bytes / size), (cuuint32_t)(kStageBytes / box_bytes), 1u};
   const cuuint32_t estr[3] = {1u, 1u, 1u};
   CUresult r = fn(m, t, 3, const_cast<void*>(in), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
                   CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
