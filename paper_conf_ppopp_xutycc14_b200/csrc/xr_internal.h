@@ -84,6 +84,7 @@ struct ColArgs {
   int64_t units;       // B * tiles * S
   int64_t G2;          // coltma: groups of kGroupFold unit partials per tile (two-level gang tier)
   int box;             // coltma: TMA box width in bytes (256, 512 or 1024; tile = box columns)
+  int packed;          // colflat, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[B*K]
   int init_from_out;
   unsigned long long* tl;  // profiling timeline (coltma; xr_debug_timeline), null when off
 };

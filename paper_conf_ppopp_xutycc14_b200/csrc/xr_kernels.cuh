@@ -878,6 +878,13 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
     const Acc* col = reinterpret_cast<const Acc*>(red);  // col[c], c < K
     if (a.S == 1) {
       for (int c = t; c < a.K; c += kBlock) out[b * a.K + c] = merge_init<OP, T>(col[c], out, b * a.K + c, a.init_from_out);
+    } else if (PackedAdd<OP, T>::value && a.packed) {  // a4 in one atomic per column (32-bit int '+')
+      unsigned long long* pk = reinterpret_cast<unsigned long long*>(a.tickets) + b * a.K;
+      for (int c = t; c < a.K; c += kBlock) {
+        uint32_t sum;
+        if (packed_add_arrive(pk + c, (uint32_t)col[c], a.S, &sum))
+          out[b * a.K + c] = merge_init<OP, T>((Acc)sum, out, b * a.K + c, a.init_from_out);
+      }
     } else {
       // a4, two levels over the S unit partial rows of batch b (K values each)
       Acc* P1 = partials + b * a.S * a.K;                         // [S][K]

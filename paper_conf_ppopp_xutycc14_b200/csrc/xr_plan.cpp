@@ -180,11 +180,18 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       p->splits = S;
       p->units = B * S;
       p->group = kBlock;
+      ColArgs& c = p->col;
       if (S > 1) {
         p->ws_bytes = B * (S + G2) * K * asz;
         p->tickets = B * (G2 + 1);
+        // 32-bit integer '+': one packed (sum, count) word per output column
+        // instead of partial rows and two ticket levels (xr_ops.cuh PackedAdd)
+        if (op == XR_OP_ADD && dtype == XR_INT32 && env.get("XR_NO_PACKED") == nullptr) {
+          p->ws_bytes = 0;
+          p->tickets = 2 * B * K;
+          c.packed = 1;
+        }
       }
-      ColArgs& c = p->col;
       c.B = B; c.R = R; c.K = K; c.tiles = 1; c.S = S; c.units = p->units; c.G2 = G2;
       return;
     }

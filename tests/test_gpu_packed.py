@@ -87,3 +87,28 @@ def test_packed_graph_replay():
         g.replay()
         torch.cuda.synchronize()
         check("+", "int32", dims, lv, out.cpu().numpy(), x)
+
+
+# flat column kernel (RK / KRK with narrow rows): one packed word per output column
+FLAT = [
+    ((64, 64, 128), "gw"),           # cfg1 testsuite nest at gang + worker
+    ((1 << 20, 2, 32), "g"),         # the paper's 2^20 x 2 x 32 gang case: 1184 splits per column
+    ((3000, 1, 64), "g"),
+    ((9, 4000, 32), "w"),            # KRK: 9 batches
+    ((100000, 1, 4), "g"),           # 16-B rows
+]
+
+
+@pytest.mark.parametrize("dims,lv", FLAT)
+def test_packed_colflat_int32_sum(dims, lv):
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    p = _plan(xr, dims, lv)
+    assert p["kernel"] == "colflat" and p["splits"] > 1, p
+    assert p["tickets"] == 2 * p["out_count"] and p["ws_bytes"] == 0, p
+    n = int(np.prod(dims))
+    x = datagen.uniform_int(6161 + n % 89, n, -(1 << 31), (1 << 31) - 1, np.int32)
+    got = gpu_reduce("+", "int32", dims, lv, x)
+    check("+", "int32", dims, lv, got, x)
+    assert np.array_equal(got, gpu_reduce("+", "int32", dims, lv, x))  # self-reset
+    init = datagen.uniform_int(98, p["out_count"], -(1 << 31), (1 << 31) - 1, np.int32)
+    check("+", "int32", dims, lv, gpu_reduce("+", "int32", dims, lv, x, init=init), x, init=init)
