@@ -159,8 +159,11 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     // small inputs): the flat column kernel streams whole rows contiguously.
     const int64_t row_bytes = K * size;
     const bool pow2 = (row_bytes & (row_bytes - 1)) == 0;
+    const char* efm = env.get("XR_FLAT_MAX_ROW");  // A/B: widest row (bytes) for large inputs
+    const int64_t flat_max = efm ? std::atoll(efm) : 512;
     if (!seg_only && aligned && pow2 && row_bytes >= 16 &&
-        (row_bytes <= 512 || (seg_only_small && row_bytes <= 4096)) && env.get("XR_NO_FLAT") == nullptr) {
+        (row_bytes <= std::min<int64_t>(flat_max, 4096) || (seg_only_small && row_bytes <= 4096)) &&
+        env.get("XR_NO_FLAT") == nullptr) {
       const int64_t rp4k = 4096 / row_bytes;
       const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch
       const char* eu = env.get("XR_FLAT_UNITS_PER_CTA");  // tuning overrides
