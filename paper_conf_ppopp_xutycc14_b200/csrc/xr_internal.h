@@ -66,6 +66,7 @@ struct SegArgs {
   int64_t units;       // O * S
   int init_from_out;
   int packed;            // seg kernel, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[O]
+  int smaj;              // stream kernel, RKR: unit ids split-major (else output-major)
   int use_exch;          // 1: fused exchange of the O == 1 result (exch below)
   ExchArgs exch;
   unsigned long long* tl;  // profiling timeline (xr_debug_timeline), null when off
@@ -85,6 +86,7 @@ struct ColArgs {
   int64_t G2;          // coltma: groups of kGroupFold unit partials per tile (two-level gang tier)
   int box;             // coltma: TMA box width in bytes (256, 512 or 1024; tile = box columns)
   int packed;          // colflat, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[B*K]
+  int smaj;            // coltma: unit ids split-major (else tile-major)
   int init_from_out;
   unsigned long long* tl;  // profiling timeline (coltma; xr_debug_timeline), null when off
 };

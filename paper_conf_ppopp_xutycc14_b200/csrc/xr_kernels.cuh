@@ -403,8 +403,14 @@ __device__ __forceinline__ StreamGeom stream_geom(const SegArgs& a, long long u)
   StreamGeom g;
   if (a.C > 1) {  // RKR: whole 16-B aligned rows r0..r1-1 of output o (plan), no head / tail
     const int64_t S = a.Sr;
-    g.o = u / S;
-    const int64_t s = u - g.o * S;
+    int64_t s;
+    if (a.smaj) {  // split-major ids: concurrent units cover every output of one row range
+      s = u / a.O;
+      g.o = u - s * a.O;
+    } else {
+      g.o = u / S;
+      s = u - g.o * S;
+    }
     const int64_t r0 = split_lo(a.C, S, s), r1 = split_lo(a.C, S, s + 1);
     g.row = static_cast<const T*>(a.in) + g.o * a.oStride + r0 * a.rowStride;
     g.head = 0;
@@ -554,10 +560,17 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) stream_kernel(const _
       __syncwarp();
       if (lane == 0) mbar_arrive(&bfree[slot]);
       if (u < 0) break;
-      const int64_t o = u / S;
+      int64_t o, sp;  // output and split of unit u (partials stay output-major)
+      if (a.smaj && a.C > 1) {
+        sp = u / a.O;
+        o = u - sp * a.O;
+      } else {
+        o = u / S;
+        sp = u - o * S;
+      }
       unsigned t = 0;
       if (lane == 0) {
-        partials[u] = v;
+        partials[o * S + sp] = v;
         t = ticket_add(&a.tickets[o]);
       }
       t = __shfl_sync(0xffffffffu, t, 0);
@@ -1497,6 +1510,23 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
   const int64_t per_b = a.tiles * a.S;
+  // unit id -> (batch, tile, split): tile-major (the splits of one tile are
+  // consecutive ids) or split-major (a.smaj: concurrently claimed units cover
+  // every tile of the same row range -- one moving window of the array)
+  auto decode = [&](long long u, int64_t* b, int64_t* tile, int64_t* s) {
+    if (a.smaj) {
+      const int64_t bt = a.B * a.tiles;
+      *s = u / bt;
+      const int64_t r = u - *s * bt;
+      *b = r / a.tiles;
+      *tile = r - *b * a.tiles;
+    } else {
+      *b = u / per_b;
+      const int64_t rem = u - *b * per_b;
+      *tile = rem / a.S;
+      *s = rem - *tile * a.S;
+    }
+  };
 
   if (tid0 == 0) {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmap)) : "memory");
@@ -1529,8 +1559,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
           mbar_arrive(&full[slot0]);
           break;
         }
-        const int64_t b = u / per_b, rem = u - b * per_b;
-        const int64_t tile = rem / a.S, s = rem - tile * a.S;
+        int64_t b, tile, s;
+        decode(u, &b, &tile, &s);
         int64_t r0, r1;
         box_rows(a.R, a.S, s, BR, &r0, &r1);
         const int64_t nk = (r1 - r0 + BR - 1) / BR;
@@ -1597,8 +1627,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
   long long pend_u = -1;   // the pending unit (uniform across consumers)
   auto finish_pending = [&]() {
     if (pend_u < 0) return;
-    const int64_t b = pend_u / per_b, rem = pend_u - b * per_b;
-    const int64_t tile = rem / a.S, s = rem - tile * a.S;
+    int64_t b, tile, s;
+    decode(pend_u, &b, &tile, &s);
     const int64_t tid_tile = b * a.tiles + tile;
     const int64_t grp_i = s / kGroupFold;
     const int64_t g0 = grp_i * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
@@ -1637,8 +1667,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
     const long long u = s_units[seq & (RING - 1)];
     if (u < 0) break;
-    const int64_t b = u / per_b, rem = u - b * per_b;
-    const int64_t tile = rem / a.S, s = rem - tile * a.S;
+    int64_t b, tile, s;
+    decode(u, &b, &tile, &s);
     int64_t r0, r1;
     box_rows(a.R, a.S, s, BR, &r0, &r1);
     const int64_t nk = (r1 - r0 + BR - 1) / BR;

@@ -264,6 +264,9 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       }
       ColArgs& c = p->col;
       c.B = B; c.R = R; c.K = K; c.tiles = tiles; c.S = S; c.units = p->units; c.G2 = G2; c.box = box;
+      // split-major unit ids (r02ah same-process A/B: cfg3 columns 613.7 ->
+      // 597.8 us, cfg5 GW -0.6 to -1.7 %; S == 1 plans are unaffected)
+      c.smaj = env.get("XR_COLTMA_TILE_MAJOR") == nullptr ? 1 : 0;
       return;
     }
     const int64_t TW = 32 * cv;
@@ -453,6 +456,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   SegArgs& s = p->seg;
   s.O = O; s.C = C; s.L = L; s.rowStride = rowStride; s.oStride = oStride;
   s.Sr = Sr; s.Sc = Sc; s.units = p->units;
+  s.smaj = (stream && C > 1 && env.get("XR_STREAM_SPLIT_MAJOR") != nullptr) ? 1 : 0;  // A/B
 
   // Guided units for the whole-array stream (R shape): per-CTA timelines
   // (tools/timeline.py) showed the equal-unit tail -- the CTAs finish over
