@@ -29,10 +29,29 @@ cases = [
     ("+", "int32", (64, 64, 128), "g"),           # colsmall (r02)
     ("max", "fp64", (40, 33, 100), "w"),          # colsmall KRK, half-width last group
 ]
+# r02: packed (sum, count) gang tier of the seg and flat column kernels
+cases += [
+    ("+", "int32", (64, 64, 128), "gwv"),         # seg W=CTA, packed, one unit per CTA
+    ("+", "int32", (64, 64, 128), "gv"),          # seg W=32, packed
+    ("+", "int32", (3000, 1, 64), "g"),           # colflat, packed
+]
+# staged kernels on small inputs (XR_SMALL_BYTES=0): column TMA kernel with
+# 256-B boxes + split-major units (8-byte split tiles), 1 KiB boxes, rkr
+staged = [
+    ("*", "fp64", (4096, 1, 512), "g"),           # coltma, 256-B boxes, S > 1, split-major
+    ("&&", "fp32", (700, 1, 512), "g"),           # coltma, 1 KiB boxes, S > 1
+    ("^", "int64", (2000, 3, 512), "w"),          # coltma KRK, S == 1
+    ("max", "int32", (40, 64, 256), "gv"),        # rkr
+]
+KIND = {"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "^": "bxor", "&&": "land", "|": "bor"}
 for op, dtype, dims, lv in cases:
-    x = recipes.make({"+": "ints", "*": "mul", "max": "maxmin", "min": "maxmin", "^": "bxor", "&&": "land",
-                      "|": "bor"}[op], dims, oracle.mask_of(lv), dtype, 1)
+    x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, 1)
     check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
+os.environ["XR_SMALL_BYTES"] = "0"
+for op, dtype, dims, lv in staged:
+    x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, 1)
+    check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x), x)
+del os.environ["XR_SMALL_BYTES"]
 # heat (bulk + register variants), transform-reduce, multi, paper kernels
 for nj, ni in [(70, 1030), (33, 67), (9, 5), (41, 1027)]:  # odd ni: shifted bulk staging (clip at the buffer end)
     T0 = oracle.heat_init(nj, ni)
