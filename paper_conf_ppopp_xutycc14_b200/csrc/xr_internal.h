@@ -87,11 +87,15 @@ struct ColArgs {
   int box;             // coltma: TMA box width in bytes (256, 512 or 1024; tile = box columns)
   int packed;          // colflat, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[B*K]
   int smaj;            // coltma: unit ids split-major (else tile-major)
+  int gf;              // coltma: unit partials per group of the two-level gang tier
   int init_from_out;
   unsigned long long* tl;  // profiling timeline (coltma; xr_debug_timeline), null when off
 };
 
-constexpr int kGroupFold = 64;  // unit partials folded per group by the group's last CTA
+#ifndef XR_GROUP_FOLD
+#define XR_GROUP_FOLD 64
+#endif
+constexpr int kGroupFold = XR_GROUP_FOLD;  // unit partials folded per group by the group's last CTA
 
 // Elementwise: out[o] = init (+) in[o] (ident) or out[o] = init (fill).
 struct EltArgs {

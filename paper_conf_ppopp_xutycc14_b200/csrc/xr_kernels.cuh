@@ -1614,7 +1614,7 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     }
     return z;
   };
-  // a4, two levels: unit partial -> group of kGroupFold (its last unit folds
+  // a4, two levels: unit partial -> group of a.gf (its last unit folds
   // the group in unit order) -> tile (the last group folds the G2 group
   // partials).  The group ticket of a unit is DEFERRED: consumer thread 0
   // issues the fence + atomic after the unit's partial store and the
@@ -1630,8 +1630,8 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
     int64_t b, tile, s;
     decode(pend_u, &b, &tile, &s);
     const int64_t tid_tile = b * a.tiles + tile;
-    const int64_t grp_i = s / kGroupFold;
-    const int64_t g0 = grp_i * kGroupFold, gsz = min((int64_t)kGroupFold, a.S - g0);
+    const int64_t grp_i = s / a.gf;
+    const int64_t g0 = grp_i * a.gf, gsz = min((int64_t)a.gf, a.S - g0);
     if (tid == 0) s_last = (pend_tk == (unsigned)(gsz - 1));
     cons_sync();
     pend_u = -1;
@@ -1726,7 +1726,7 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
       if (tid < TW) P1[s * TW + tid] = v;
       cons_sync();  // partial stores happen-before thread 0's (cumulative) fence; red free
       finish_pending();  // the previous unit's group (its ticket has long returned)
-      if (tid == 0) pend_tk = ticket_add(&a.tickets[tid_tile * a.G2 + s / kGroupFold]);  // result read later
+      if (tid == 0) pend_tk = ticket_add(&a.tickets[tid_tile * a.G2 + s / a.gf]);  // result read later
       pend_u = u;
 #if !XR_COLTMA_DEFER
       finish_pending();  // A/B: resolve the ticket right away (the r01 behaviour)

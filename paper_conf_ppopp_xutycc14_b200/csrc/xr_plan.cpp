@@ -256,8 +256,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       if (const char* eg = env.get("XR_COLTMA_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
       p->group = kBlock;
       p->sched = true;
-      // two-level gang tier: groups of kGroupFold unit partials, then the groups
-      const int64_t G2 = cdiv(S, kGroupFold);
+      // two-level gang tier: groups of gf unit partials, then the groups.  One
+      // group (a single level) while S <= 64; beyond, groups of 16 (r02al
+      // interleaved A/B: 32-bit GW, S = 444: 95.6 / 91.5 -> 93.8 / 88.7 us;
+      // a second level for S = 55 cost the 64-bit GW +2.3 %)
+      int gf = S <= kGroupFold ? kGroupFold : 16;
+      if (const char* eg = env.get("XR_COLTMA_GROUP")) gf = std::max(2, std::atoi(eg));  // A/B
+      const int64_t G2 = cdiv(S, gf);
       if (S > 1) {
         p->ws_bytes = B * tiles * (S + G2) * TWt * asz;
         p->tickets = B * tiles * (G2 + 1);
@@ -267,6 +272,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       // split-major unit ids (r02ah same-process A/B: cfg3 columns 613.7 ->
       // 597.8 us, cfg5 GW -0.6 to -1.7 %; S == 1 plans are unaffected)
       c.smaj = env.get("XR_COLTMA_TILE_MAJOR") == nullptr ? 1 : 0;
+      c.gf = gf;
       return;
     }
     const int64_t TW = 32 * cv;

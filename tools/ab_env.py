@@ -71,7 +71,8 @@ def main():
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
                 for _ in range(a.batch):
-                    xr.xr_reduce(op, dtype, dims, lv, x.data_ptr(), out.data_ptr(), s.cuda_stream)
+                    st = xr.xr_reduce(op, dtype, dims, lv, x.data_ptr(), out.data_ptr(), s.cuda_stream)
+                    assert st == 0, (case, name, xr.xr_strerror(st))
                 e1.record(s)
                 torch.cuda.synchronize()
                 res[name].append(e0.elapsed_time(e1) / a.batch * 1e3)

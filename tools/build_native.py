@@ -76,7 +76,7 @@ def build(force: bool = False, ptxas_verbose: bool = False, quiet: bool = True,
         obj = os.path.join(OBJ, f + ".o")
         objs.append(obj)
         if force or _stale(obj, [src] + hdr):
-            jobs.append(["g++", "-O2", "-std=c++17", "-fPIC", "-Wall", "-c", src, "-o", obj,
+            jobs.append(["g++", "-O2", "-std=c++17", "-fPIC", "-Wall", *["-D" + d for d in defines], "-c", src, "-o", obj,
                          "-I", os.path.join(CUDA, "include"), *inc])
     if jobs:
         with cf.ThreadPoolExecutor(max_workers=os.cpu_count() or 4) as ex:
