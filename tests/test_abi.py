@@ -228,3 +228,18 @@ def test_shard_plan_init_merged_once(xr):
     assert xr.xr_shard_plan("+", "fp32", (8, 2, 2), "g", 2, 0)["merge_init"] == 0
     with pytest.raises(xr.XReduceError):
         xr.xr_shard_plan("+", "fp32", (8, 2, 2), "g", 2, 2)
+
+
+def test_plan_column_box_group_rules(xr):
+    """Column TMA plans (DESIGN 6.0, r02 A/B): 8-byte split tiles take 256-B
+    boxes (16 tiles of 32 columns for 512 kept fp64 columns), 4-byte ones
+    1 KiB boxes (2 tiles of 256 fp32 columns); one gang-tier level while
+    S <= 64 (tickets = tiles * 2), groups of 16 beyond (S = 444: 28 groups)."""
+    p = xr.xr_plan_describe("*", "fp64", (512, 512, 512), "gw", 256)
+    assert p["kernel"] == "coltma" and p["splits"] == 55 and p["units"] == 16 * 55
+    assert p["tickets"] == 16 * 2
+    q = xr.xr_plan_describe("*", "int32", (512, 512, 512), "gw", 256)
+    assert q["kernel"] == "coltma" and q["splits"] == 444 and q["units"] == 2 * 444
+    assert q["tickets"] == 2 * (28 + 1)
+    r = xr.xr_plan_describe("*", "fp64", (512, 512, 512), "g", 256)  # whole-tile units, 1 KiB boxes
+    assert r["kernel"] == "coltma" and r["splits"] == 1 and r["units"] == 262144 // 128

@@ -463,3 +463,31 @@ def test_stream_rkr_rows(dtype, row_bytes, splits, monkeypatch):
         if dtype.startswith("int"):  # & | ^ on the same path
             xb = recipes.make("bxor", dims, oracle.mask_of("gv"), dtype, R1 + K)
             check("^", dtype, dims, "gv", gpu_reduce("^", dtype, dims, "gv", xb), xb)
+
+
+@pytest.mark.parametrize("box", ["256", "512", "1024"])
+@pytest.mark.parametrize("order", ["split", "tile"])
+@pytest.mark.parametrize("group", ["auto", "3"])
+def test_coltma_box_order_group(box, order, group, monkeypatch):
+    """The column TMA kernel's round-2 variants on ragged RK / KRK shapes, every
+    dtype: TMA box width (256 / 512 / 1024 B x 16 KiB), split-major or
+    tile-major unit ids, and the two-level gang tier with groups of 3 unit
+    partials (many groups per tile, so the second level always runs), with
+    init; each plan is checked to be the column TMA kernel with the forced
+    settings."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    monkeypatch.setenv("XR_COLTMA_BOX", box)
+    if order == "tile":
+        monkeypatch.setenv("XR_COLTMA_TILE_MAJOR", "1")
+    if group != "auto":
+        monkeypatch.setenv("XR_COLTMA_GROUP", group)
+    cases = [("+", "fp32", (999, 1, 1000), "g"), ("max", "int32", (3, 301, 640), "w"),
+             ("*", "fp64", (700, 1, 260), "g"), ("^", "int64", (2, 257, 1030), "w"),
+             ("&&", "fp32", (4100, 1, 384), "g")]
+    for op, dtype, dims, lv in cases:
+        p = xr.xr_plan_describe(op, dtype, dims, lv, 256)
+        assert p["kernel"] == "coltma", (dims, p)
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, sum(dims) + int(box))
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 5)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
