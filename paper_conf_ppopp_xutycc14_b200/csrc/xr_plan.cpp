@@ -312,11 +312,18 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   else { O = run_n[1]; C = run_n[0]; L = run_n[2]; rowStride = O * L; oStride = L; p->shape = XR_SHAPE_RKR; }
 
   const int64_t row_bytes = L * size;
+  // RKR with 2-4 KiB rows and at least as many reduced rows per output as
+  // outputs (C >= O: few outputs, long strided columns of rows) run faster on
+  // the register seg kernel's finer units than on the ring kernels (r02aq
+  // interleaved A/B over 12 shapes: C >= O 3-8 % faster on seg, C <= O / 4
+  // 2-6 % slower; 1 KiB and 512 B rows stay on rkr, 6-81 % faster there).
+  const bool rkr_to_seg = nr == 3 && row_bytes >= 2048 && row_bytes <= 4096 && C >= O &&
+                          env.get("XR_RKR_RING") == nullptr;
   // RKR with short rows (power-of-two row_bytes in [512 B, 2 KiB], 16-B
   // aligned, at least one full 16 KiB j-block): the rkr rows kernel -- units
   // are (block of J = 16 KiB / row_bytes outputs, range of k), each stage one
   // bulk copy of J contiguous rows, accumulated per warp in registers.
-  if (!seg_only && !seg_only_small && nr == 3 && row_bytes >= 512 && row_bytes <= 2048 &&
+  if (!seg_only && !seg_only_small && !rkr_to_seg && nr == 3 && row_bytes >= 512 && row_bytes <= 2048 &&
       (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= kStageBytes / row_bytes &&
       env.get("XR_NO_RKR") == nullptr && env.get("XR_NO_BULK") == nullptr) {
     const int64_t J = kStageBytes / row_bytes;
@@ -418,7 +425,7 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // (4 KiB rows) 0.95-1.01 of peak vs 0.66-0.95 for the seg kernel; 32-bit
   // (2 KiB rows) no better than seg (0.83-0.87 both), so those stay on seg.
   const char* rkr_min = env.get("XR_RKR_STREAM_MIN_ROW");  // tuning override (bytes)
-  const bool rkr_stream = nr == 3 && row_bytes >= (rkr_min ? std::atoll(rkr_min) : 4096) &&
+  const bool rkr_stream = nr == 3 && !rkr_to_seg && row_bytes >= (rkr_min ? std::atoll(rkr_min) : 4096) &&
                           row_bytes % 16 == 0 && in_addr % 16 == 0 && env.get("XR_NO_RKR_STREAM") == nullptr;
   const bool stream = !seg_only && !seg_only_small && env.get("XR_NO_BULK") == nullptr &&
                       ((C == 1 && row_bytes >= (int64_t)kStages * kStageBytes) || rkr_stream);

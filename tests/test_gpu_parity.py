@@ -423,6 +423,7 @@ def test_rkr_kernel_short_rows(dtype, row_bytes, units, monkeypatch):
     CTA (few long units) to 64, with init."""
     import paper_conf_ppopp_xutycc14_b200 as xr
     monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    monkeypatch.setenv("XR_RKR_RING", "1")  # C >= O with 2 KiB rows would take the seg kernel
     if units != "auto":
         monkeypatch.setenv("XR_RKR_UNITS_PER_CTA", units)
     L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
@@ -451,6 +452,7 @@ def test_stream_rkr_rows(dtype, row_bytes, splits, monkeypatch):
     monkeypatch.setenv("XR_SMALL_BYTES", "0")
     monkeypatch.setenv("XR_RKR_STREAM_MIN_ROW", "1024")  # the planner's default is 4 KiB rows
     monkeypatch.setenv("XR_NO_RKR", "1")  # 1-2 KiB rows would take the rkr rows kernel
+    monkeypatch.setenv("XR_RKR_RING", "1")  # C >= O with 2-4 KiB rows would take the seg kernel
     if splits != "auto":
         monkeypatch.setenv("XR_STREAM_SPLITS", splits)
     L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
