@@ -1816,13 +1816,18 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       auto kern = stream_kernel<OP, T, XR_STREAM_NS, kStageBytes>;
       constexpr int dyn = XR_STREAM_NS * kStageBytes;
       int occ = occ_dev<stream_kernel<OP, T, XR_STREAM_NS, kStageBytes>>(kWsEpiBlock, dyn);
-      // 2 resident CTAs per SM (r02 same-box A/B vs 3: 2^30 fp32 584.2 vs
-      // 588.1 us, 32768^2 rows 578.5 vs 582.0, 512^3 64-bit GV 156.2 vs 158.2,
-      // 32-bit WV 82.5 vs 84.4; 0.5-1 GiB whole arrays equal; 64-bit GWV
-      // 160.2 vs 158.2).  XR_STREAM_CTAS_PER_SM overrides.
+      // Resident CTAs per SM by unit length: 3 for units < 128 KiB, else 2.
+      // Short units must stream longer than a claim round trip (~1.5-2 us)
+      // to hide it, so they want the slower per-CTA rate of 3 CTAs per SM
+      // (r02au / r02av interleaved A/B: 512 MiB whole arrays, 64 KiB units,
+      // 91.4 -> 81.2 us; 1 GiB fp64, 113 KiB units, 163.7 -> 155.4; 16-256 MiB
+      // 3-10 % faster); long units keep 2 (2^30 fp32, 453 KiB units, 583.7 vs
+      // 585.5; 32768^2 rows, 128 KiB units, 578.5 vs 582.0; 256 KiB KR units
+      // level).  XR_STREAM_CTAS_PER_SM overrides.
       {
+        const int64_t unit_bytes = p.seg.O * p.seg.C * p.seg.L * (int64_t)sizeof(T) / std::max<int64_t>(p.units, 1);
         const char* e = std::getenv("XR_STREAM_CTAS_PER_SM");
-        occ = std::max(1, std::min(occ, e ? std::atoi(e) : 2));
+        occ = std::max(1, std::min(occ, e ? std::atoi(e) : unit_bytes < (int64_t(128) << 10) ? 3 : 2));
       }
       if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid_for(p.units, num_sms, occ)), dim3(kWsEpiBlock), dyn, s,
                                      p.seg))

@@ -110,11 +110,11 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // Small inputs are latency bound, not bandwidth bound: the staged (bulk /
   // TMA ring) kernels would run on a few dozen CTAs, so below kSmallBytes the
   // register kernels, which spread one load round over many CTAs, are used.
+  const char* sb = env.get("XR_SMALL_BYTES");  // test / tuning override
+  const int64_t small = sb ? std::atoll(sb) : kSmallBytes;
   {
     int64_t total = 1;
     for (int d = 0; d < 3; ++d) total *= dims[d];
-    const char* sb = env.get("XR_SMALL_BYTES");  // test / tuning override
-    const int64_t small = sb ? std::atoll(sb) : kSmallBytes;
     if (total * size < small) seg_only_small = true;
   }
 
@@ -198,8 +198,16 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
       c.B = B; c.R = R; c.K = K; c.tiles = 1; c.S = S; c.units = p->units; c.G2 = G2;
       return;
     }
-    // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31
-    if (!seg_only && !seg_only_small && aligned && K * size >= 1024 && R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
+    // TMA path: 16-B aligned rows of >= 1 KiB (one box row), R < 2^31, inputs
+    // of >= 48 MiB (r02av: the register column kernel is 22-30 % faster at
+    // 16-32 MiB, the TMA kernel 12-16 % faster from 64 MiB)
+    // (an explicit XR_SMALL_BYTES below that also lowers it: the tests' way
+    // of running the staged kernels on small, ragged shapes)
+    const char* ecm = env.get("XR_COLTMA_MIN_BYTES");
+    const int64_t coltma_min = ecm ? std::atoll(ecm) : sb ? std::min<int64_t>(small, int64_t(48) << 20)
+                                                          : (int64_t(48) << 20);
+    if (!seg_only && !seg_only_small && aligned && K * size >= 1024 && B * R * K * size >= coltma_min &&
+        R < (int64_t(1) << 31) && K < (int64_t(1) << 31) &&
         B < (int64_t(1) << 31) && env.get("XR_NO_TMA") == nullptr && !no_tma) {
       // Balance (measured r01 sweeps): the producer warp keeps every CTA's ring
       // full, so few long units per CTA are best, but the unit count must be an
@@ -376,7 +384,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     p->splits = 1;
     p->units = units;
     p->sched = true;
-    p->grid_hint = std::min<int64_t>(cap, cdiv(units, k));
+    // every resident CTA while each keeps >= 4 stages (its ring full): the r01
+    // grid of units / k left 16-256 MiB inputs on 32-256 CTAs (r02av: 16 MiB
+    // of 2 KiB rows 29 us vs 8.4 on the register kernel)
+    p->grid_hint = std::min<int64_t>(cap, std::max<int64_t>(cdiv(units, k), cdiv(nst, 4)));
     if (const char* eg = env.get("XR_ROWS_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
     SegArgs& s = p->seg;
     s.O = O; s.C = 1; s.L = L; s.rowStride = 0; s.oStride = L;

@@ -115,7 +115,7 @@ def test_tma_encode_failure_falls_back(monkeypatch):
     onto the register column kernel (one launch) and stays correct."""
     import torch
     import paper_conf_ppopp_xutycc14_b200 as xr
-    dims = (1, 4096, 2048)
+    dims = (1, 4096, 4096)  # 64 MiB: above the column TMA kernel's 48 MiB threshold
     x = datagen.uniform_int(5, int(np.prod(dims)), -(1 << 20), 1 << 20, np.int32)
     xd = torch.from_numpy(x).cuda()
     assert xr.xr_plan_describe("+", "int32", dims, "w", xd.data_ptr())["kernel"] == "coltma"
