@@ -41,6 +41,8 @@ def main():
     ap.add_argument("--cfg", action="append", required=True, help="NAME:VAR=VAL,VAR=VAL (NAME: for defaults)")
     ap.add_argument("--rounds", type=int, default=7)
     ap.add_argument("--batch", type=int, default=10)
+    ap.add_argument("--single", action="store_true",
+                    help="time each launch alone (events around it, synchronised: no overlap with the next launch)")
     a = ap.parse_args()
     cfgs = [parse_cfg(c) for c in a.cfg]
     keys = sorted({k for _, e in cfgs for k in e})
@@ -68,6 +70,18 @@ def main():
             order = cfgs if r % 2 == 0 else cfgs[::-1]
             for name, env in order:
                 setenv(env)
+                if a.single:
+                    ts = []
+                    for _ in range(a.batch):
+                        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        e0.record(s)
+                        st = xr.xr_reduce(op, dtype, dims, lv, x.data_ptr(), out.data_ptr(), s.cuda_stream)
+                        assert st == 0, (case, name, xr.xr_strerror(st))
+                        e1.record(s)
+                        torch.cuda.synchronize()
+                        ts.append(e0.elapsed_time(e1) * 1e3)
+                    res[name].append(statistics.median(ts))
+                    continue
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(s)
                 for _ in range(a.batch):
