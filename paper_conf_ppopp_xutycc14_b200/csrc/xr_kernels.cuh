@@ -1008,7 +1008,26 @@ __device__ __forceinline__ void rkr_unit(int64_t u, int64_t S, int64_t njb, int6
 #endif
 }
 
-template <int OP, typename T, int NS>
+// NARROW rows (16-256 B, r02): a stage holds J = 64-1024 rows, so consumer
+// thread ct meets vectors ct + 256 i (i < 4) of every stage -- rows
+// ct / vpr + i * (256 / vpr), always the same 4 outputs, piece ct % vpr --
+// and accumulates them in registers across the k range; at the unit end the
+// vpr threads of a row combine by shuffles and the row's leader runs the
+// per-output gang tier itself (partial, ticket; the warp folds the outputs
+// whose last split it holds).  The seg kernel read such rows 16-256 B at a
+// time at the k stride: 0.7-1.5 TB/s (r02az).
+template <typename Acc, int OP, typename T>
+__device__ __forceinline__ Acc narrow_row_reduce(Acc v, int vpr) {
+  switch (vpr) {
+    case 1: return v;
+    case 2: return group_reduce<OP, T, 2>(v);
+    case 4: return group_reduce<OP, T, 4>(v);
+    case 8: return group_reduce<OP, T, 8>(v);
+    default: return group_reduce<OP, T, 16>(v);
+  }
+}
+
+template <int OP, typename T, int NS, bool NARROW>
 __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __grid_constant__ RkrArgs a) {
   using O = Op<OP, T>;
   using Acc = typename O::Acc;
@@ -1084,6 +1103,101 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   }
 
   Acc* partials = static_cast<Acc*>(a.partials);
+  if constexpr (NARROW) {
+    if (warp == kConsWarps + 1) return;  // the consumers run the gang tier
+    const int ct = tid - 32;
+    const int vpr = (int)(row_bytes >> 4);  // 16-B vectors per row: 1..16
+    const int rstep = kConsThreads / vpr;   // rows between my 4 vectors of a stage
+    const int rb = ct / vpr;                // my first row of every stage
+    const bool leader = (ct & (vpr - 1)) == 0;
+    int seq = 0;
+    int64_t g = 0;
+    while (true) {
+      mbar_wait(&full[g % NS], (unsigned)((g / NS) & 1));
+      const long long u = s_units[seq & (RING - 1)];
+      if (u < 0) break;
+      int64_t jb, s;
+      rkr_unit(u, S, a.units / S, &jb, &s);
+      const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
+      const int nrows = (int)min((int64_t)J, a.K - jb * J);
+      Acc acc[4][VEC];
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) acc[i][q] = O::identity();
+      for (int64_t k = k0; k < k1; ++k, ++g) {
+        const int slot = (int)(g % NS);
+        if (k > k0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
+        const unsigned char* sm = stage_mem + slot * STAGE;
+        if (nrows == J) {  // all 4 shared-memory loads in flight, then fold
+          U128 x[4];
+#pragma unroll
+          for (int i = 0; i < 4; ++i) x[i] = *reinterpret_cast<const U128*>(sm + (ct + i * kConsThreads) * 16);
+#pragma unroll
+          for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) acc[i][q] = O::combine(acc[i][q], O::lift(unpack<T>(x[i], q)));
+        } else {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            if (rb + i * rstep < nrows) {
+              const U128 x = *reinterpret_cast<const U128*>(sm + (ct + i * kConsThreads) * 16);
+#pragma unroll
+              for (int q = 0; q < VEC; ++q) acc[i][q] = O::combine(acc[i][q], O::lift(unpack<T>(x, q)));
+            }
+          }
+        }
+        fence_proxy_async_smem();  // generic reads before the async refill
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[slot]);
+      }
+      // my 4 rows: combine, then (S > 1) store all 4 partials, ONE fence, and
+      // the 4 tickets in flight together (one round trip, not four)
+      Acc v[4];
+      unsigned tk[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        v[i] = acc[i][0];
+#pragma unroll
+        for (int q = 1; q < VEC; ++q) v[i] = O::combine(v[i], acc[i][q]);
+        v[i] = narrow_row_reduce<Acc, OP, T>(v[i], vpr);  // the row's vpr threads (lanes of one warp)
+        const int r = rb + i * rstep;
+        const int64_t o = jb * J + r;
+        if (leader && r < nrows) {
+          if (S == 1) out[o] = merge_init<OP, T>(v[i], out, o, a.init_from_out);
+          else partials[o * S + s] = v[i];
+        }
+      }
+      if (S > 1) {
+        __threadfence();
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (leader && rb + i * rstep < nrows) tk[i] = atomicAdd(&a.tickets[jb * J + rb + i * rstep], 1u);
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        if (S == 1) break;
+        const int r = rb + i * rstep;
+        const int64_t o = jb * J + r;
+        const bool last = leader && r < nrows && tk[i] == (unsigned)(S - 1);
+        unsigned m = __ballot_sync(0xffffffffu, last);
+        if (m) __threadfence();
+        while (m) {  // the warp folds each output whose last split it holds, in split order
+          const int l = __ffs(m) - 1;
+          m &= m - 1;
+          const int64_t ol = __shfl_sync(0xffffffffu, o, l);
+          Acc w = fold_partials<OP, T>(partials + ol * S, S, lane, 32);
+          w = group_reduce<OP, T, 32>(w);
+          if (lane == 0) {
+            out[ol] = merge_init<OP, T>(w, out, ol, a.init_from_out);
+            a.tickets[ol] = 0u;
+          }
+        }
+      }
+      ++seq;
+    }
+    return;
+  }
   if (warp == kConsWarps + 1) {
     // ---------------- epilogue warp (a4 per output, as in stream_kernel): lane
     // r takes row r's unit value, writes the partial and the output's ticket;
@@ -1835,12 +1949,15 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       break;
     }
     case K_RKR: {
-      auto kern = rkr_kernel<OP, T, kStages>;
       constexpr int dyn = kStages * kStageBytes;
-      const int occ = occ_dev<rkr_kernel<OP, T, kStages>>(kWsEpiBlock, dyn);
+      const bool narrow = p.rkr.L * (int64_t)sizeof(T) < 512;
+      const int occ = narrow ? occ_dev<rkr_kernel<OP, T, kStages, true>>(kWsEpiBlock, dyn)
+                             : occ_dev<rkr_kernel<OP, T, kStages, false>>(kWsEpiBlock, dyn);
       int64_t grid = grid_for(p.units, num_sms, occ);
       if (p.grid_hint > 0) grid = std::min(grid, p.grid_hint);
-      if (cudaError_t e = launch_pdl(kern, dim3((unsigned)grid), dim3(kWsEpiBlock), dyn, s, p.rkr)) return e;
+      if (cudaError_t e = narrow ? launch_pdl(rkr_kernel<OP, T, kStages, true>, dim3((unsigned)grid), dim3(kWsEpiBlock), dyn, s, p.rkr)
+                                 : launch_pdl(rkr_kernel<OP, T, kStages, false>, dim3((unsigned)grid), dim3(kWsEpiBlock), dyn, s, p.rkr))
+        return e;
       break;
     }
     case K_ROWS: {

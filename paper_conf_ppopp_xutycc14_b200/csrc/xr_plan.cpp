@@ -331,7 +331,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // aligned, at least one full 16 KiB j-block): the rkr rows kernel -- units
   // are (block of J = 16 KiB / row_bytes outputs, range of k), each stage one
   // bulk copy of J contiguous rows, accumulated per warp in registers.
-  if (!seg_only && !seg_only_small && !rkr_to_seg && nr == 3 && row_bytes >= 512 && row_bytes <= 2048 &&
+  // narrow rows (16-256 B, r02): rkr_kernel's NARROW consumers (4 fixed rows
+  // per thread per stage); the seg kernel read them at 0.7-1.5 TB/s
+  const bool rkr_narrow = row_bytes >= 16 && row_bytes < 512 && env.get("XR_NO_RKR_NARROW") == nullptr;
+  if (!seg_only && !seg_only_small && !rkr_to_seg && nr == 3 && (rkr_narrow || row_bytes >= 512) && row_bytes <= 2048 &&
       (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= kStageBytes / row_bytes &&
       env.get("XR_NO_RKR") == nullptr && env.get("XR_NO_BULK") == nullptr) {
     const int64_t J = kStageBytes / row_bytes;
@@ -343,7 +346,8 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     // k units per resident CTA, each >= kStages stages (k values)
     int64_t S = std::max<int64_t>(1, std::min<int64_t>(cdiv(k * cap, njb), C / kStages));
     // fp32 '+': each lane accumulator folds vpl elements per k (chains <= kChainCap)
-    if (chain_capped) S = std::max<int64_t>(S, cdiv(C * (row_bytes >> 9), (int64_t)kChainCap));
+    // (narrow rows: one element per accumulator per k)
+    if (chain_capped) S = std::max<int64_t>(S, cdiv(C * std::max<int64_t>(1, row_bytes >> 9), (int64_t)kChainCap));
     S = std::max<int64_t>(1, std::min<int64_t>(S, C));
     p->kernel = K_RKR;
     p->group = 32;
@@ -353,7 +357,10 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     p->sched = true;
     // 2 CTAs per SM (r02 grid sweep, 512^3 32-bit GV: 88.5 us at 222 / 296
     // CTAs vs 90.4-91.5 us at 444)
-    p->grid_hint = std::min<int64_t>((int64_t)std::max(num_sms, 1) * 2, p->units);
+    // narrow rows: every resident CTA (r02bb A/B: 3 / SM 1-5 % faster; their
+    // consumers run the per-output tier themselves, a unit end is costlier)
+    const int64_t per_sm = row_bytes < 512 ? 3 : 2;
+    p->grid_hint = std::min<int64_t>((int64_t)std::max(num_sms, 1) * per_sm, p->units);
     if (const char* eg = env.get("XR_RKR_GRID")) p->grid_hint = std::max(1, std::atoi(eg));  // A/B
     if (S > 1) {
       p->ws_bytes = O * S * asz;

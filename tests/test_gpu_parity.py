@@ -493,3 +493,32 @@ def test_coltma_box_order_group(box, order, group, monkeypatch):
         x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, sum(dims) + int(box))
         init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 5)
         check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [16, 32, 64, 128, 256])
+@pytest.mark.parametrize("units", ["auto", "1", "16"])
+def test_rkr_narrow_rows(dtype, row_bytes, units, monkeypatch):
+    """RKR with NARROW rows (16-256 B): the rkr kernel's narrow consumers (each
+    thread meets the same 4 rows of every 16 KiB stage, rows combined by
+    shuffles, the row leaders run the per-output gang tier), forced with
+    XR_SMALL_BYTES=0; ragged j-blocks (outputs not a multiple of the J =
+    16 KiB / row_bytes rows of a stage), k split from 1 unit per CTA to 16,
+    with init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    if units != "auto":
+        monkeypatch.setenv("XR_RKR_UNITS_PER_CTA", units)
+    L = row_bytes // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    J = 16384 // row_bytes
+    for R1, K, op in [(7, J, "+"), (33, J + 5, "max"), (5, 2 * J + 1, "&&"), (64, J, "*"), (19, 3 * J - 7, "||"),
+                      (1, J, "min")]:
+        dims = (R1, K, L)
+        x = recipes.make(KIND[op], dims, oracle.mask_of("gv"), dtype, R1 * K + row_bytes)
+        init = recipes.make("ints", (K, 1, 1), 1, dtype, 4)
+        check(op, dtype, dims, "gv", gpu_reduce(op, dtype, dims, "gv", x, init=init), x, init=init)
+        if R1 > 1:
+            assert xr.xr_plan_describe(op, dtype, dims, "gv", 256)["kernel"] == "rkr"
+        if dtype.startswith("int"):
+            xb = recipes.make("bxor", dims, oracle.mask_of("gv"), dtype, R1 + K)
+            check("^", dtype, dims, "gv", gpu_reduce("^", dtype, dims, "gv", xb), xb)
