@@ -67,6 +67,7 @@ struct SegArgs {
   int init_from_out;
   int packed;            // seg kernel, 32-bit int '+': packed (sum, count) gang tier, tickets = u64[O]
   int smaj;              // stream kernel, RKR: unit ids split-major (else output-major)
+  int seg_static;        // seg kernel, CTA-wide units: static round-robin assignment (no claims)
   int use_exch;          // 1: fused exchange of the O == 1 result (exch below)
   ExchArgs exch;
   unsigned long long* tl;  // profiling timeline (xr_debug_timeline), null when off

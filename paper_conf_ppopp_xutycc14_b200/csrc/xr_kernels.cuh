@@ -283,13 +283,16 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
     __shared__ long long s_unit[2];
     // one unit per CTA (small, latency-bound inputs): static assignment, no
     // claim round trip at the start and no exit counter at the end
+    // a.seg_static (A/B): every CTA takes units blockIdx.x + i * gridDim.x,
+    // no claims at all
     const bool one_each = a.units <= (int64_t)gridDim.x;
-    if (threadIdx.x == 0) s_unit[0] = one_each ? (long long)blockIdx.x : claim_first(a.sched);
+    const bool stat = one_each || a.seg_static;
+    if (threadIdx.x == 0) s_unit[0] = stat ? (long long)blockIdx.x : claim_first(a.sched);
     __syncthreads();
     long long u = s_unit[0];
     int par = 1;
     while (u < a.units) {
-      if (threadIdx.x == 0) s_unit[par] = one_each ? (long long)a.units : claim_next(a.sched);  // next, in flight
+      if (threadIdx.x == 0) s_unit[par] = stat ? u + (long long)gridDim.x : claim_next(a.sched);  // next, in flight
       int64_t o;
       Acc v = seg_unit<OP, T, W, U>(a, u, threadIdx.x, &o);
       v = block_reduce<OP, T, BLOCK>(v, smem);  // a2 + a3
@@ -330,7 +333,7 @@ __global__ void __launch_bounds__(BLOCK, XR_SEG_MINB) seg_kernel(const __grid_co
       u = s_unit[par];
       par ^= 1;
     }
-    if (!one_each) sched_exit(a.sched);
+    if (!stat) sched_exit(a.sched);
   } else {
     static_assert(W <= 32 && (32 % W) == 0, "sub-warp group");
     const int lane = threadIdx.x & (W - 1);

@@ -488,6 +488,12 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   s.O = O; s.C = C; s.L = L; s.rowStride = rowStride; s.oStride = oStride;
   s.Sr = Sr; s.Sc = Sc; s.units = p->units;
   s.smaj = (stream && C > 1 && env.get("XR_STREAM_SPLIT_MAJOR") != nullptr) ? 1 : 0;  // A/B
+  // CTA-wide seg units without splits (KR rows of 4-64 KiB): static
+  // round-robin units, no claim round trip per unit (r02bc interleaved A/B:
+  // 16 KiB rows 58.7 -> 50.4 us, 8 KiB rows -5.5 %; with splits and tickets
+  // the dynamic claims stay, static was 12 % slower there)
+  s.seg_static = (!stream && W == kBlock && S == 1 && p->units >= 4 * target_ctas) ? 1 : 0;
+  if (const char* es = env.get("XR_SEG_STATIC")) s.seg_static = std::atoi(es) != 0 ? 1 : 0;  // A/B
 
   // Guided units for the whole-array stream (R shape): per-CTA timelines
   // (tools/timeline.py) showed the equal-unit tail -- the CTAs finish over
