@@ -421,7 +421,14 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     s.Sr = 1; s.Sc = kClusterCtas; s.units = kClusterCtas;
     return;
   }
-  int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= 4096 ? 32 : kBlock;
+  // warp groups for rows up to 64 KiB (longer rows take the stream kernel):
+  // r02bd interleaved A/B, 512 MiB of 8 KiB rows 168.8 -> 78.8 us (fp64 173.0
+  // -> 78.8), 16 KiB rows 95.5 -> 79.0, 32 KiB rows 106.0 -> 54.0 (256 MiB)
+  // against CTA-wide groups (r01 limit 4 KiB); one 256 MiB case of 16 KiB
+  // rows was 6 % slower
+  const char* ew = env.get("XR_SEG_W32_MAX");  // A/B: widest row (bytes) for warp groups
+  const int64_t w32_max = ew ? std::atoll(ew) : 65536;
+  int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= w32_max ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
   const int64_t work = C * L;  // elements per output
