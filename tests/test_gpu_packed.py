@@ -19,7 +19,7 @@ pytestmark = pytest.mark.gpu
 # (dims, mask, seg group width) -- plans checked below to be packed seg plans
 CASES = [
     ((64, 64, 128), "gwv", 256),     # cfg1 testsuite nest: one unit per CTA
-    ((64, 64, 128), "wv", 256),      # two CTA splits per output
+    ((64, 64, 128), "wv", 32),       # 32 KiB rows: warp groups, 16 splits per output
     ((64, 64, 128), "gv", 32),       # warp groups, 16 splits per output
     ((1, 1, 3000001), "gwv", 256),   # ragged whole array
     ((33, 1, 77777), "v", 256),      # long ragged rows split per CTA
