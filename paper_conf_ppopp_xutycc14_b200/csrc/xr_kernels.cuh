@@ -839,7 +839,11 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
   const int t = threadIdx.x;
   const int64_t row_bytes = a.K * (int64_t)sizeof(T);
   const int G = (int)(row_bytes >> 4);            // 16-B column groups per row (1..256)
-  const int64_t rp4k = 4096 / row_bytes;           // rows per 4 KiB load round
+  const int64_t rp4k = 4096 / row_bytes;           // whole rows per (<= 4 KiB) load round
+  // vectors per round (r02: rows of any multiple of 16 B, not only powers of
+  // two): a round is rp4k whole rows, so thread t < NV always meets column
+  // group t % G; threads >= NV idle (<= 6 % of the CTA)
+  const int NV = (int)(rp4k * G);
   const int64_t nblk = (a.R + rp4k - 1) / rp4k;    // 4 KiB row blocks per batch
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
@@ -853,17 +857,17 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
     for (int k = 0; k < U; ++k)
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[k][q] = O::identity();
-    int64_t v = t;
-    for (; v + (int64_t)(U - 1) * kBlock < nv; v += (int64_t)U * kBlock) {
+    int64_t v = t < NV ? t : nv;
+    for (; v + (int64_t)(U - 1) * NV < nv; v += (int64_t)U * NV) {
       U128 x[U];
 #pragma unroll
-      for (int k = 0; k < U; ++k) x[k] = ld_stream(base + v + (int64_t)k * kBlock);
+      for (int k = 0; k < U; ++k) x[k] = ld_stream(base + v + (int64_t)k * NV);
 #pragma unroll
       for (int k = 0; k < U; ++k)
 #pragma unroll
         for (int q = 0; q < VEC; ++q) acc[k][q] = O::combine(acc[k][q], O::lift(unpack<T>(x[k], q)));
     }
-    for (; v < nv; v += kBlock) {
+    for (; v < nv; v += NV) {
       const U128 x = ld_stream(base + v);
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], O::lift(unpack<T>(x, q)));
@@ -881,7 +885,7 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
     if (t < G) {
 #pragma unroll
       for (int q = 0; q < VEC; ++q) w[q] = red[t][q];
-      for (int m = t + G; m < kBlock; m += G)
+      for (int m = t + G; m < NV; m += G)
 #pragma unroll
         for (int q = 0; q < VEC; ++q) w[q] = O::combine(w[q], red[m][q]);
     }

@@ -161,8 +161,11 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     const bool pow2 = (row_bytes & (row_bytes - 1)) == 0;
     const char* efm = env.get("XR_FLAT_MAX_ROW");  // A/B: widest row (bytes) for large inputs
     const int64_t flat_max = efm ? std::atoll(efm) : 512;
-    if (!seg_only && aligned && pow2 && row_bytes >= 16 &&
-        (row_bytes <= std::min<int64_t>(flat_max, 4096) || (seg_only_small && row_bytes <= 4096)) &&
+    // (r02: any multiple of 16 B -- rounds of whole rows -- and non-power-of-
+    // two rows below 1 KiB, which the TMA column kernel does not take)
+    const bool flat_width = row_bytes <= std::min<int64_t>(flat_max, 4096) || (seg_only_small && row_bytes <= 4096) ||
+                            (!pow2 && row_bytes < 1024 && env.get("XR_NO_FLAT_NPOW2") == nullptr);
+    if (!seg_only && aligned && (pow2 || env.get("XR_NO_FLAT_NPOW2") == nullptr) && row_bytes >= 16 && flat_width &&
         env.get("XR_NO_FLAT") == nullptr) {
       const int64_t rp4k = 4096 / row_bytes;
       const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch
