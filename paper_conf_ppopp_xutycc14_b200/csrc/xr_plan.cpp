@@ -431,7 +431,14 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // rows was 6 % slower
   const char* ew = env.get("XR_SEG_W32_MAX");  // A/B: widest row (bytes) for warp groups
   const int64_t w32_max = ew ? std::atoll(ew) : 65536;
-  int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= 128 ? 8 : row_bytes <= w32_max ? 32 : kBlock;
+  // 8-lane groups for KR rows below 4 KiB (four rows per warp in flight):
+  // r02bh / r02bi interleaved A/B, 512 MiB of 500 / 1000 / 2000 / 3000 B rows
+  // 348 / 176 / 101 / 92 -> 123 / 95 / 84 / 85 us, the 2 MiB cfg1 v nest
+  // (512 B rows) 1.96 -> 1.62 us per graph-replayed call; RKR segments and
+  // 4 KiB rows stay on 32 lanes (16-38 % and 2 % slower on 8)
+  const char* ew8 = env.get("XR_SEG_W8_MAX");  // A/B: widest row (bytes) for 8-lane groups
+  const int64_t w8_max = ew8 ? std::atoll(ew8) : C == 1 ? 4095 : 128;
+  int W = (seg_only && !sub_cta) ? kBlock : row_bytes <= w8_max ? 8 : row_bytes <= w32_max ? 32 : kBlock;
   auto resident_groups = [&](int w) { return target_ctas * (kBlock / w); };
   auto min_unit_elems = [&](int w) { return (int64_t)w * vec * kUnroll; };
   const int64_t work = C * L;  // elements per output
