@@ -1054,8 +1054,8 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   T* out = static_cast<T*>(a.out);
   const int64_t row_bytes = a.L * (int64_t)sizeof(T);
-  const int rshift = __ffsll(row_bytes) - 1;  // row_bytes is a power of two
-  const int J = (int)(STAGE >> rshift);        // rows (outputs) per stage: 8, 16 or 32
+  const int rshift = __ffsll(row_bytes) - 1;  // row_bytes is a power of two (except NARROW rows)
+  const int J = (int)(STAGE / row_bytes);      // rows (outputs) per stage: 8, 16 or 32 (NARROW: 64..1024)
   const int64_t S = a.S;                       // k splits per j-block
 
   if (tid == 0) {
@@ -1093,9 +1093,9 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
         int64_t jb, s;
         rkr_unit(u, S, a.units / S, &jb, &s);
         const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
-        const unsigned nb = (unsigned)(min((int64_t)J, a.K - jb * J) << rshift);
-        const char* src = static_cast<const char*>(a.in) + ((k0 * a.K + jb * J) << rshift);
-        const int64_t kstride = a.K << rshift;  // bytes between consecutive k
+        const unsigned nb = (unsigned)(min((int64_t)J, a.K - jb * J) * row_bytes);
+        const char* src = static_cast<const char*>(a.in) + (k0 * a.K + jb * J) * row_bytes;
+        const int64_t kstride = a.K * row_bytes;  // bytes between consecutive k
         for (int64_t k = k0; k < k1; ++k, ++g, src += kstride) {
           const int slot = (int)(g % NS);
           if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
@@ -1113,10 +1113,16 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   if constexpr (NARROW) {
     if (warp == kConsWarps + 1) return;  // the consumers run the gang tier
     const int ct = tid - 32;
-    const int vpr = (int)(row_bytes >> 4);  // 16-B vectors per row: 1..16
-    const int rstep = kConsThreads / vpr;   // rows between my 4 vectors of a stage
-    const int rb = ct / vpr;                // my first row of every stage
-    const bool leader = (ct & (vpr - 1)) == 0;
+    const int vpr = (int)(row_bytes >> 4);  // 16-B vectors per row: 1..31
+    // power-of-two rows: a row's vpr vectors sit in consecutive lanes of one
+    // warp (shuffle combine); other multiples of 16 B: through shared memory
+    const bool shfl = (vpr & (vpr - 1)) == 0;
+    __shared__ Acc nsm[kConsThreads * 4];   // per-vector unit values (non-power-of-two rows)
+    const int nvec = J * vpr;               // vectors of a full stage (<= 1024)
+    int rowi[4];                            // row of my vector i of every stage
+#pragma unroll
+    for (int i = 0; i < 4; ++i) rowi[i] = (ct + i * kConsThreads) / vpr;
+    const bool leader = shfl && (ct & (vpr - 1)) == 0;
     int seq = 0;
     int64_t g = 0;
     while (true) {
@@ -1136,7 +1142,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
         const int slot = (int)(g % NS);
         if (k > k0) mbar_wait(&full[slot], (unsigned)((g / NS) & 1));
         const unsigned char* sm = stage_mem + slot * STAGE;
-        if (nrows == J) {  // all 4 shared-memory loads in flight, then fold
+        if (nrows == J && nvec == 4 * kConsThreads) {  // all 4 shared-memory loads in flight, then fold
           U128 x[4];
 #pragma unroll
           for (int i = 0; i < 4; ++i) x[i] = *reinterpret_cast<const U128*>(sm + (ct + i * kConsThreads) * 16);
@@ -1147,7 +1153,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
         } else {
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
-            if (rb + i * rstep < nrows) {
+            if (ct + i * kConsThreads < nvec && rowi[i] < nrows) {
               const U128 x = *reinterpret_cast<const U128*>(sm + (ct + i * kConsThreads) * 16);
 #pragma unroll
               for (int q = 0; q < VEC; ++q) acc[i][q] = O::combine(acc[i][q], O::lift(unpack<T>(x, q)));
@@ -1159,34 +1165,61 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
         if (lane == 0) mbar_arrive(&empty[slot]);
       }
       // my 4 rows: combine, then (S > 1) store all 4 partials, ONE fence, and
-      // the 4 tickets in flight together (one round trip, not four)
+      // the 4 tickets in flight together (one round trip, not four).  Power-
+      // of-two rows: the row's vpr lanes combine by shuffles and the leader
+      // lane owns the row; other rows: every vector's value goes to shared
+      // memory and thread ct owns rows ct + 256 i, folding their vpr vectors
+      // in order.
       Acc v[4];
       unsigned tk[4];
+      int orow[4];      // the row thread ct owns in slot i, or -1
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
         v[i] = acc[i][0];
 #pragma unroll
         for (int q = 1; q < VEC; ++q) v[i] = O::combine(v[i], acc[i][q]);
-        v[i] = narrow_row_reduce<Acc, OP, T>(v[i], vpr);  // the row's vpr threads (lanes of one warp)
-        const int r = rb + i * rstep;
-        const int64_t o = jb * J + r;
-        if (leader && r < nrows) {
-          if (S == 1) out[o] = merge_init<OP, T>(v[i], out, o, a.init_from_out);
-          else partials[o * S + s] = v[i];
+      }
+      if (shfl) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          v[i] = narrow_row_reduce<Acc, OP, T>(v[i], vpr);  // the row's vpr threads (lanes of one warp)
+          orow[i] = (leader && rowi[i] < nrows) ? rowi[i] : -1;
         }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+          if (ct + i * kConsThreads < nvec) nsm[ct + i * kConsThreads] = v[i];
+        cons_sync();
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int r = ct + i * kConsThreads;
+          orow[i] = r < nrows ? r : -1;
+          if (r < nrows) {
+            Acc w = nsm[r * vpr];
+            for (int p2 = 1; p2 < vpr; ++p2) w = O::combine(w, nsm[r * vpr + p2]);
+            v[i] = w;
+          }
+        }
+        cons_sync();  // nsm is rewritten at the next unit end
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        if (orow[i] < 0) continue;
+        const int64_t o = jb * J + orow[i];
+        if (S == 1) out[o] = merge_init<OP, T>(v[i], out, o, a.init_from_out);
+        else partials[o * S + s] = v[i];
       }
       if (S > 1) {
         __threadfence();
 #pragma unroll
         for (int i = 0; i < 4; ++i)
-          if (leader && rb + i * rstep < nrows) tk[i] = atomicAdd(&a.tickets[jb * J + rb + i * rstep], 1u);
+          if (orow[i] >= 0) tk[i] = atomicAdd(&a.tickets[jb * J + orow[i]], 1u);
       }
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
         if (S == 1) break;
-        const int r = rb + i * rstep;
-        const int64_t o = jb * J + r;
-        const bool last = leader && r < nrows && tk[i] == (unsigned)(S - 1);
+        const int64_t o = jb * J + (orow[i] >= 0 ? orow[i] : 0);
+        const bool last = orow[i] >= 0 && tk[i] == (unsigned)(S - 1);
         unsigned m = __ballot_sync(0xffffffffu, last);
         if (m) __threadfence();
         while (m) {  // the warp folds each output whose last split it holds, in split order

@@ -334,11 +334,13 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
   // aligned, at least one full 16 KiB j-block): the rkr rows kernel -- units
   // are (block of J = 16 KiB / row_bytes outputs, range of k), each stage one
   // bulk copy of J contiguous rows, accumulated per warp in registers.
-  // narrow rows (16-256 B, r02): rkr_kernel's NARROW consumers (4 fixed rows
-  // per thread per stage); the seg kernel read them at 0.7-1.5 TB/s
+  // narrow rows (16-496 B, multiples of 16 B, r02): rkr_kernel's NARROW
+  // consumers (4 fixed rows per thread per stage); the seg kernel read them
+  // at 0.7-1.5 TB/s
   const bool rkr_narrow = row_bytes >= 16 && row_bytes < 512 && env.get("XR_NO_RKR_NARROW") == nullptr;
   if (!seg_only && !seg_only_small && !rkr_to_seg && nr == 3 && (rkr_narrow || row_bytes >= 512) && row_bytes <= 2048 &&
-      (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 && O >= kStageBytes / row_bytes &&
+      ((row_bytes & (row_bytes - 1)) == 0 || (rkr_narrow && row_bytes % 16 == 0)) && in_addr % 16 == 0 &&
+      O >= kStageBytes / row_bytes &&
       env.get("XR_NO_RKR") == nullptr && env.get("XR_NO_BULK") == nullptr) {
     const int64_t J = kStageBytes / row_bytes;
     const int64_t njb = cdiv(O, J);

@@ -496,12 +496,14 @@ def test_coltma_box_order_group(box, order, group, monkeypatch):
 
 
 @pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
-@pytest.mark.parametrize("row_bytes", [16, 32, 64, 128, 256])
+@pytest.mark.parametrize("row_bytes", [16, 32, 64, 128, 256, 48, 80, 240, 496])
 @pytest.mark.parametrize("units", ["auto", "1", "16"])
 def test_rkr_narrow_rows(dtype, row_bytes, units, monkeypatch):
-    """RKR with NARROW rows (16-256 B): the rkr kernel's narrow consumers (each
-    thread meets the same 4 rows of every 16 KiB stage, rows combined by
-    shuffles, the row leaders run the per-output gang tier), forced with
+    """RKR with NARROW rows (16-496 B; powers of two and other multiples of
+    16 B): the rkr kernel's narrow consumers (each thread meets the same 4
+    rows of every stage of whole rows; rows combined by shuffles, or through
+    shared memory when a row's vectors straddle warps; the row owners run the
+    per-output gang tier), forced with
     XR_SMALL_BYTES=0; ragged j-blocks (outputs not a multiple of the J =
     16 KiB / row_bytes rows of a stage), k split from 1 unit per CTA to 16,
     with init."""
