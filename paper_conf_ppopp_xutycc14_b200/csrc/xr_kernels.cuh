@@ -1055,7 +1055,7 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
   T* out = static_cast<T*>(a.out);
   const int64_t row_bytes = a.L * (int64_t)sizeof(T);
   const int rshift = __ffsll(row_bytes) - 1;  // row_bytes is a power of two (except NARROW rows)
-  const int J = (int)(STAGE / row_bytes);      // rows (outputs) per stage: 8, 16 or 32 (NARROW: 64..1024)
+  const int J = NARROW ? (int)(STAGE / row_bytes) : (int)(STAGE >> rshift);  // rows (outputs) per stage: 8, 16 or 32 (NARROW: 64..1024)
   const int64_t S = a.S;                       // k splits per j-block
 
   if (tid == 0) {
@@ -1093,9 +1093,12 @@ __global__ void __launch_bounds__(kWsEpiBlock, XR_WS_MINB) rkr_kernel(const __gr
         int64_t jb, s;
         rkr_unit(u, S, a.units / S, &jb, &s);
         const int64_t k0 = split_lo(a.C, S, s), k1 = split_lo(a.C, S, s + 1);
-        const unsigned nb = (unsigned)(min((int64_t)J, a.K - jb * J) * row_bytes);
-        const char* src = static_cast<const char*>(a.in) + (k0 * a.K + jb * J) * row_bytes;
-        const int64_t kstride = a.K * row_bytes;  // bytes between consecutive k
+        // (NARROW rows need not be powers of two: multiply; the others shift)
+        const unsigned nb = NARROW ? (unsigned)(min((int64_t)J, a.K - jb * J) * row_bytes)
+                                   : (unsigned)(min((int64_t)J, a.K - jb * J) << rshift);
+        const char* src = static_cast<const char*>(a.in) +
+                          (NARROW ? (k0 * a.K + jb * J) * row_bytes : (k0 * a.K + jb * J) << rshift);
+        const int64_t kstride = NARROW ? a.K * row_bytes : a.K << rshift;  // bytes between consecutive k
         for (int64_t k = k0; k < k1; ++k, ++g, src += kstride) {
           const int slot = (int)(g % NS);
           if (g >= NS) mbar_wait(&empty[slot], (unsigned)(((g / NS) - 1) & 1));
@@ -1893,6 +1896,53 @@ __global__ void __launch_bounds__(kWsBlock, XR_WS_MINB) coltma_kernel(const __gr
   if (tid == 0) tl_event(a.tl, TL_END, 0);
 }
 
+// ------------------------------------------------------------- short-row kernel
+// KR with SHORT power-of-two rows (4-128 B, 16-B aligned input; r02): every
+// thread takes one CH-byte chunk (CH = max(64 B, row)) of whole rows per
+// round -- CH / 16 vector loads in flight -- folds each row in element order
+// and writes its CH / row_bytes outputs; adjacent threads hold adjacent
+// chunks, so loads and stores are coalesced.  The seg kernel's 8-lane groups
+// reduced one such row per group and round: 8 B rows at 0.14 TB/s (r02bk).
+template <int OP, typename T, int CH>
+__global__ void __launch_bounds__(kBlock) shortrow_kernel(const __grid_constant__ SegArgs a) {
+  pdl_wait();  // no global access above this line
+  pdl_trigger();
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / (int)sizeof(T);
+  constexpr int NVC = CH / 16;                 // vectors per chunk
+  constexpr int E = CH / (int)sizeof(T);       // elements per chunk
+  const T* in = static_cast<const T*>(a.in);
+  T* out = static_cast<T*>(a.out);
+  const int L = (int)a.L;                      // elements per row (power of two, <= E)
+  const int rpt = E / L;                       // rows per chunk
+  const int64_t nchunks = a.O / rpt;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  for (int64_t c = t0; c < nchunks; c += stride) {
+    const U128* p = reinterpret_cast<const U128*>(in + c * E);
+    U128 x[NVC];
+#pragma unroll
+    for (int v = 0; v < NVC; ++v) x[v] = ld_stream(p + v);
+    Acc acc = O::identity();
+#pragma unroll
+    for (int e = 0; e < E; ++e) {
+      acc = O::combine(acc, O::lift(unpack<T>(x[e / VEC], e % VEC)));
+      if (((e + 1) & (L - 1)) == 0) {  // row e / L complete
+        const int64_t o = c * rpt + e / L;
+        out[o] = merge_init<OP, T>(acc, out, o, a.init_from_out);
+        acc = O::identity();
+      }
+    }
+  }
+  // rows of the last partial chunk: one thread per row, in element order
+  for (int64_t o = nchunks * rpt + t0; o < a.O; o += stride) {
+    Acc acc = O::identity();
+    for (int i = 0; i < L; ++i) acc = O::combine(acc, O::lift(ld_scalar(in + o * L + i)));
+    out[o] = merge_init<OP, T>(acc, out, o, a.init_from_out);
+  }
+}
+
 // ------------------------------------------------------------- elementwise
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
@@ -2044,6 +2094,18 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       attr[1].val.clusterDim.y = 1;
       attr[1].val.clusterDim.z = 1;
       if (cudaError_t e = cudaLaunchKernelEx(&cfg, kern, p.seg)) return e;
+      break;
+    }
+    case K_SHORTROW: {
+      const int64_t row_bytes = p.seg.L * (int64_t)sizeof(T);
+      const int64_t work = (p.seg.O * row_bytes + 63) / 64;  // 64-B chunks
+      if (row_bytes > 64) {
+        const int occ = occ_dev<shortrow_kernel<OP, T, 128>>(kBlock, 0);
+        if (cudaError_t e = launch_pdl(shortrow_kernel<OP, T, 128>, dim3((unsigned)grid_for((work + 2 * kBlock - 1) / (2 * kBlock), num_sms, occ)), dim3(kBlock), 0, s, p.seg)) return e;
+      } else {
+        const int occ = occ_dev<shortrow_kernel<OP, T, 64>>(kBlock, 0);
+        if (cudaError_t e = launch_pdl(shortrow_kernel<OP, T, 64>, dim3((unsigned)grid_for((work + kBlock - 1) / kBlock, num_sms, occ)), dim3(kBlock), 0, s, p.seg)) return e;
+      }
       break;
     }
     case K_COLSMALL: {

@@ -375,6 +375,20 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     r.K = O; r.L = L; r.C = C; r.S = S; r.units = p->units;
     return;
   }
+  // SHORT contiguous rows (KR, row_bytes a power of two in [4 B, 128 B],
+  // 16-B aligned): a thread per 64 / 128-B chunk of whole rows (shortrow_kernel)
+  if (!seg_only && nr == 2 && row_bytes <= 128 && (row_bytes & (row_bytes - 1)) == 0 && in_addr % 16 == 0 &&
+      env.get("XR_NO_SHORTROW") == nullptr) {
+    p->kernel = K_SHORTROW;
+    p->group = 1;
+    p->vec = vec;
+    p->splits = 1;
+    p->units = O;
+    SegArgs& s = p->seg;
+    s.O = O; s.C = 1; s.L = L; s.rowStride = 0; s.oStride = L;
+    s.Sr = 1; s.Sc = 1; s.units = O;
+    return;
+  }
   // short contiguous rows (KR, row_bytes a power of two in [512 B, 2 KiB],
   // 16-B aligned): whole rows streamed in blocks of 16 KiB stages (rows_kernel)
   if (!seg_only && !seg_only_small && nr == 2 && row_bytes >= 512 && row_bytes <= 2048 &&

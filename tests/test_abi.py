@@ -128,7 +128,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
     assert p["kernel"] in (("col", "coltma", "colflat", "colsmall") if shape in ("RK", "KRK")
-                           else ("seg", "stream", "rows", "rkr"))
+                           else ("seg", "stream", "rows", "rkr", "shortrow"))
 
 
 def test_plan_canonical_cfg2_cfg3_cfg5(xr):

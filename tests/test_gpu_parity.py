@@ -524,3 +524,28 @@ def test_rkr_narrow_rows(dtype, row_bytes, units, monkeypatch):
         if dtype.startswith("int"):
             xb = recipes.make("bxor", dims, oracle.mask_of("gv"), dtype, R1 + K)
             check("^", dtype, dims, "gv", gpu_reduce("^", dtype, dims, "gv", xb), xb)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("row_bytes", [8, 16, 32, 64, 128])
+def test_shortrow_kernel(dtype, row_bytes):
+    """KR with short power-of-two rows (8-128 B): the short-row kernel (a thread
+    per 64 / 128-B chunk of whole rows, rows folded in element order), every
+    op, row counts that leave a partial last chunk, with init; a misaligned
+    start takes the seg kernel instead (checked too)."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    size = np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    if row_bytes < 2 * size:
+        pytest.skip("a row of one element is not a reduction")
+    L = row_bytes // size
+    for O, op in [(1, "+"), (7, "max"), (1000, "*"), (4099, "&&"), (65537, "||"), (333, "min")]:
+        dims = (O, 1, L)
+        x = recipes.make(KIND[op], dims, oracle.mask_of("v"), dtype, O + row_bytes)
+        init = recipes.make("ints", (O, 1, 1), 1, dtype, 3)
+        if O > 1:  # one row is the whole-array (R) shape
+            assert xr.xr_plan_describe(op, dtype, dims, "v", 256)["kernel"] == "shortrow"
+        check(op, dtype, dims, "v", gpu_reduce(op, dtype, dims, "v", x, init=init), x, init=init)
+        check(op, dtype, dims, "v", gpu_reduce(op, dtype, dims, "v", x, offset=1), x)
+        if dtype.startswith("int"):
+            xb = recipes.make("bxor", dims, oracle.mask_of("v"), dtype, O)
+            check("^", dtype, dims, "v", gpu_reduce("^", dtype, dims, "v", xb), xb)

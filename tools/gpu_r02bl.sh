@@ -1,0 +1,7 @@
+#!/bin/bash
+# r02bl: short-row kernel -- parity + A/B vs the seg kernel
+O=gpurun_out/r02bl; mkdir -p $O
+timeout 900 python -m pytest tests/test_gpu_parity.py -q -x -k "shortrow or all_pairs or fuzz or init_from_out or cfg1" > $O/pytest.log 2>&1; echo "pytest rc=$?" >> $O/pytest.log
+tail -n 2 $O/pytest.log
+timeout 1200 python tools/ab_env.py --cases nest-add-fp32-1024x65536x2-v nest-add-fp32-524288x16x16-v nest-add-fp32-4096x1024x32-v nest-max-int32-16x524288x16-v nest-mul-fp64-67108864x1x2-v nest-add-fp64-4194304x1x16-v \
+  --cfg A: --cfg seg:XR_NO_SHORTROW=1 --rounds 5 --batch 5 2>&1 | tee $O/ab_shortrow.jsonl
