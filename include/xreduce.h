@@ -244,7 +244,8 @@ typedef struct {
                            9 rkr (bulk-streamed j-blocks of short rows, k loop),
                            10 colsmall (warp per 32 B of columns, small inputs),
                            11 rcluster (one 16-CTA cluster, DSMEM gang tier),
-                           12 shortrow (thread per chunk of short rows) */
+                           12 shortrow (thread per chunk of short rows),
+                           13 thincol (thread per column group, few rows) */
   int64_t cdims[3];     /* canonical extents (shape-dependent, rest 0)       */
   int64_t out_count;
   int group;            /* seg: lanes per group (8, 32 or the CTA size)      */

@@ -31,7 +31,7 @@ GANG, WORKER, VECTOR, INIT_FROM_OUT = 0x1, 0x2, 0x4, 0x100
 OK, ERR_INVALID, ERR_UNSUPPORTED, ERR_CUDA, ERR_NCCL, ERR_NOMEM = range(6)
 SHAPES = {0: "none", 1: "fill", 2: "ident", 3: "R", 4: "KR", 5: "RK", 6: "KRK", 7: "RKR"}
 KERNELS = {0: "none", 1: "fill", 2: "ident", 3: "seg", 4: "col", 5: "stream", 6: "coltma", 7: "rows", 8: "colflat", 9: "rkr",
-           10: "colsmall", 11: "rcluster", 12: "shortrow"}
+           10: "colsmall", 11: "rcluster", 12: "shortrow", 13: "thincol"}
 COLL_NONE, COLL_ALLREDUCE, COLL_ALLGATHER_COMBINE, COLL_ALLGATHER = range(4)
 
 OPS = {"+": OP_ADD, "*": OP_MUL, "max": OP_MAX, "min": OP_MIN, "&": OP_BAND, "|": OP_BOR,

@@ -13,7 +13,7 @@ constexpr int kChainCap = 4096; // max sequential fp32 '+' chain per accumulator
 constexpr int kTargetCtasPerSm = 8;  // 2048 threads/SM at 256 threads/CTA
 constexpr int kUnitsPerCta = 8;      // dynamic units per resident CTA (tail balance)
 
-enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6, K_ROWS = 7, K_COLFLAT = 8, K_RKR = 9, K_COLSMALL = 10, K_RCLUSTER = 11, K_SHORTROW = 12 };
+enum Kernel : int { K_NONE = 0, K_FILL = 1, K_IDENT = 2, K_SEG = 3, K_COL = 4, K_STREAM = 5, K_COLTMA = 6, K_ROWS = 7, K_COLFLAT = 8, K_RKR = 9, K_COLSMALL = 10, K_RCLUSTER = 11, K_SHORTROW = 12, K_THINCOL = 13 };
 constexpr int kClusterCtas = 16;  // rcluster_kernel: one thread-block cluster (non-portable size)
 constexpr int kClusterBlock = 1024;
 

@@ -1943,6 +1943,52 @@ __global__ void __launch_bounds__(kBlock) shortrow_kernel(const __grid_constant_
   }
 }
 
+// ------------------------------------------------------------- thin column kernel
+// RK / KRK with FEW reduced rows (R <= 32) and many kept columns, 16-B
+// aligned rows (r02): the output is as large as the input, so each thread
+// owns one 16-B column group, folds its R rows in order (4 loads in flight)
+// and stores VEC outputs -- an elementwise-style pass.  The column kernels'
+// tiles and splits cost a full unit per 2-16 rows there (r02bk: R = 2 rows
+// of 256 MiB in 874 us).
+template <int OP, typename T>
+__global__ void __launch_bounds__(kBlock) thincol_kernel(const __grid_constant__ ColArgs a) {
+  pdl_wait();  // no global access above this line
+  pdl_trigger();
+  using O = Op<OP, T>;
+  using Acc = typename O::Acc;
+  constexpr int VEC = 16 / (int)sizeof(T);
+  const T* in = static_cast<const T*>(a.in);
+  T* out = static_cast<T*>(a.out);
+  const int64_t gpr = a.K / VEC;  // 16-B column groups per row
+  const int64_t ng = a.B * gpr;
+  const int R = (int)a.R;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < ng; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t b = c / gpr, cg = c - b * gpr;
+    const T* base = in + b * a.R * a.K + cg * VEC;
+    Acc acc[VEC];
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) acc[q] = O::identity();
+    int r = 0;
+    for (; r + 3 < R; r += 4) {
+      U128 x[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) x[k] = ld_stream(base + (int64_t)(r + k) * a.K);
+#pragma unroll
+      for (int k = 0; k < 4; ++k)
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) acc[q] = O::combine(acc[q], O::lift(unpack<T>(x[k], q)));
+    }
+    for (; r < R; ++r) {
+      const U128 x = ld_stream(base + (int64_t)r * a.K);
+#pragma unroll
+      for (int q = 0; q < VEC; ++q) acc[q] = O::combine(acc[q], O::lift(unpack<T>(x, q)));
+    }
+    const int64_t o = b * a.K + cg * VEC;
+#pragma unroll
+    for (int q = 0; q < VEC; ++q) out[o + q] = merge_init<OP, T>(acc[q], out, o + q, a.init_from_out);
+  }
+}
+
 // ------------------------------------------------------------- elementwise
 template <int OP, typename T>
 __global__ void __launch_bounds__(kBlock) ident_kernel(EltArgs a) {
@@ -2094,6 +2140,12 @@ cudaError_t launch_typed(Plan& p, int num_sms, cudaStream_t s) {
       attr[1].val.clusterDim.y = 1;
       attr[1].val.clusterDim.z = 1;
       if (cudaError_t e = cudaLaunchKernelEx(&cfg, kern, p.seg)) return e;
+      break;
+    }
+    case K_THINCOL: {
+      const int occ = occ_dev<thincol_kernel<OP, T>>(kBlock, 0);
+      const int64_t ng = p.col.B * p.col.K / (16 / (int64_t)sizeof(T));
+      if (cudaError_t e = launch_pdl(thincol_kernel<OP, T>, dim3((unsigned)grid_for((ng + kBlock - 1) / kBlock, num_sms, occ)), dim3(kBlock), 0, s, p.col)) return e;
       break;
     }
     case K_SHORTROW: {

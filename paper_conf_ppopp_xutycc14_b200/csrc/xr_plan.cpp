@@ -136,6 +136,19 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     else { B = run_n[0]; R = run_n[1]; K = run_n[2]; p->shape = XR_SHAPE_KRK; }
     const bool aligned = ((K * size) % 16 == 0) && (in_addr % 16 == 0);
     const int cv = aligned ? vec : 1;
+    // Few reduced rows (R <= 32) and many kept 16-B column groups: an
+    // elementwise-style pass, a thread per column group folding its R rows
+    // (thincol_kernel, r02bk: R = 2 was 874 us on the tiled column kernels)
+    if (!seg_only && aligned && R <= 32 && B * K / vec >= 65536 && env.get("XR_NO_THINCOL") == nullptr) {
+      p->kernel = K_THINCOL;
+      p->vec = vec;
+      p->splits = 1;
+      p->units = B * K / vec;
+      p->group = 1;
+      ColArgs& c = p->col;
+      c.B = B; c.R = R; c.K = K; c.tiles = 1; c.S = 1; c.units = p->units;
+      return;
+    }
     // seg_only (the fused multi-input / multi-variable launches): always the
     // register column decomposition below (their col_unit, xr_colunit.cuh)
     // Small inputs with few reduced rows: one warp per 32 B of kept columns

@@ -127,7 +127,7 @@ def test_plan_canonical_shapes_cfg1(xr, levels):
     shape, cd = SHAPE_TABLE[levels]
     assert p["shape"] == shape and p["cdims"] == cd
     assert p["out_count"] == oracle.out_count((64, 64, 128), levels)
-    assert p["kernel"] in (("col", "coltma", "colflat", "colsmall") if shape in ("RK", "KRK")
+    assert p["kernel"] in (("col", "coltma", "colflat", "colsmall", "thincol") if shape in ("RK", "KRK")
                            else ("seg", "stream", "rows", "rkr", "shortrow"))
 
 

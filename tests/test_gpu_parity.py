@@ -549,3 +549,22 @@ def test_shortrow_kernel(dtype, row_bytes):
         if dtype.startswith("int"):
             xb = recipes.make("bxor", dims, oracle.mask_of("v"), dtype, O)
             check("^", dtype, dims, "v", gpu_reduce("^", dtype, dims, "v", xb), xb)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "int64", "fp32", "fp64"])
+@pytest.mark.parametrize("R", [2, 3, 5, 16, 32])
+def test_thincol_kernel(dtype, R):
+    """RK / KRK with few reduced rows (R <= 32) and >= 65536 kept 16-B column
+    groups: the thin column kernel (a thread per column group folding its R
+    rows in order), every op, with init; RK and KRK (batches)."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    vec = 16 // np.dtype(oracle.NP_DTYPES[dtype]).itemsize
+    for dims, lv, op in [((R, 1, 65536 * vec), "g", "+"), ((R, 1, 65536 * vec + vec), "g", "max"),
+                         ((3, R, 32768 * vec), "w", "*"), ((R, 1, 70000 * vec), "g", "&&"), ((5, R, 16384 * vec), "w", "||")]:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, R + dims[2])
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 6)
+        assert xr.xr_plan_describe(op, dtype, dims, lv, 256)["kernel"] == "thincol", (dims, lv)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
+        if dtype.startswith("int"):
+            xb = recipes.make("bxor", dims, oracle.mask_of(lv), dtype, R)
+            check("^", dtype, dims, lv, gpu_reduce("^", dtype, dims, lv, xb), xb)
