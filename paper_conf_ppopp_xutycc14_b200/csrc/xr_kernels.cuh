@@ -838,12 +838,16 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
   __shared__ int s_last;
   const int t = threadIdx.x;
   const int64_t row_bytes = a.K * (int64_t)sizeof(T);
-  const int G = (int)(row_bytes >> 4);            // 16-B column groups per row (1..256)
+  // 8-B rows (r02: two 32-bit columns): a 16-B vector holds two whole rows,
+  // element q of every vector is column q % 2 -- one column group of VEC
+  // lanes whose lanes fold into the K columns at the end
+  const bool sub16 = row_bytes < 16;
+  const int G = sub16 ? 1 : (int)(row_bytes >> 4);  // 16-B column groups per row (1..256)
   const int64_t rp4k = 4096 / row_bytes;           // whole rows per (<= 4 KiB) load round
   // vectors per round (r02: rows of any multiple of 16 B, not only powers of
   // two): a round is rp4k whole rows, so thread t < NV always meets column
   // group t % G; threads >= NV idle (<= 6 % of the CTA)
-  const int NV = (int)(rp4k * G);
+  const int NV = (int)(rp4k * row_bytes / 16);
   const int64_t nblk = (a.R + rp4k - 1) / rp4k;    // 4 KiB row blocks per batch
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
@@ -851,7 +855,7 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
     const int64_t b = u / a.S, s = u - b * a.S;
     const int64_t r0 = min(split_lo(nblk, a.S, s) * rp4k, a.R), r1 = min(split_lo(nblk, a.S, s + 1) * rp4k, a.R);
     const U128* __restrict__ base = reinterpret_cast<const U128*>(static_cast<const T*>(a.in) + (b * a.R + r0) * a.K);
-    const int64_t nv = (r1 - r0) * (row_bytes >> 4);  // 16-B vectors of the unit
+    const int64_t nv = (r1 - r0) * row_bytes / 16;  // whole 16-B vectors of the unit
     Acc acc[U][VEC];
 #pragma unroll
     for (int k = 0; k < U; ++k)
@@ -872,6 +876,10 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
 #pragma unroll
       for (int q = 0; q < VEC; ++q) acc[0][q] = O::combine(acc[0][q], O::lift(unpack<T>(x, q)));
     }
+    if (sub16 && t == 0 && ((r1 - r0) * row_bytes) % 16 != 0) {  // an odd last 8-B row: lanes 0 .. K-1
+      const T* last = static_cast<const T*>(a.in) + (b * a.R + r1 - 1) * a.K;
+      for (int c = 0; c < (int)a.K; ++c) acc[0][c] = O::combine(acc[0][c], O::lift(ld_scalar(last + c)));
+    }
 #pragma unroll
     for (int k = 1; k < U; ++k)
 #pragma unroll
@@ -890,9 +898,15 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
         for (int q = 0; q < VEC; ++q) w[q] = O::combine(w[q], red[m][q]);
     }
     __syncthreads();
-    if (t < G) {
+    if (t < G && !sub16) {
 #pragma unroll
       for (int q = 0; q < VEC; ++q) reinterpret_cast<Acc*>(red)[t * VEC + q] = w[q];
+    } else if (t == 0 && sub16) {  // lane q holds column q % K: fold the lanes per column, in lane order
+      for (int c = 0; c < (int)a.K; ++c) {
+        Acc z = w[c];
+        for (int q = c + (int)a.K; q < VEC; q += (int)a.K) z = O::combine(z, w[q]);
+        reinterpret_cast<Acc*>(red)[c] = z;
+      }
     }
     __syncthreads();
     const Acc* col = reinterpret_cast<const Acc*>(red);  // col[c], c < K

@@ -178,7 +178,11 @@ void make_plan(int op, int dtype, const int64_t dims[3], unsigned mask, uint64_t
     // two rows below 1 KiB, which the TMA column kernel does not take)
     const bool flat_width = row_bytes <= std::min<int64_t>(flat_max, 4096) || (seg_only_small && row_bytes <= 4096) ||
                             (!pow2 && row_bytes < 1024 && env.get("XR_NO_FLAT_NPOW2") == nullptr);
-    if (!seg_only && aligned && (pow2 || env.get("XR_NO_FLAT_NPOW2") == nullptr) && row_bytes >= 16 && flat_width &&
+    // (r02: 8-B rows of two 32-bit columns too, when every batch starts 16-B
+    // aligned -- a 16-B vector then holds two whole rows)
+    const bool flat8 = row_bytes == 8 && size == 4 && in_addr % 16 == 0 && (B == 1 || (R * 8) % 16 == 0) &&
+                       env.get("XR_NO_FLAT8") == nullptr;
+    if (!seg_only && ((aligned && (pow2 || env.get("XR_NO_FLAT_NPOW2") == nullptr) && row_bytes >= 16 && flat_width) || flat8) &&
         env.get("XR_NO_FLAT") == nullptr) {
       const int64_t rp4k = 4096 / row_bytes;
       const int64_t nblk = cdiv(R, rp4k);                   // 4 KiB row blocks per batch

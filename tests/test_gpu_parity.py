@@ -568,3 +568,24 @@ def test_thincol_kernel(dtype, R):
         if dtype.startswith("int"):
             xb = recipes.make("bxor", dims, oracle.mask_of(lv), dtype, R)
             check("^", dtype, dims, lv, gpu_reduce("^", dtype, dims, lv, xb), xb)
+
+
+@pytest.mark.parametrize("dtype", ["int32", "fp32"])
+@pytest.mark.parametrize("staging", ["planned", "staged"])
+def test_colflat_two_columns(dtype, staging, monkeypatch):
+    """RK / KRK with 8-B rows (two 32-bit columns): the flat column kernel with
+    two whole rows per 16-B vector (lane q is column q % 2), odd row counts
+    (a last 8-B row folded by scalar loads), batches with an even row count,
+    every op, with init."""
+    import paper_conf_ppopp_xutycc14_b200 as xr
+    if staging == "staged":
+        monkeypatch.setenv("XR_SMALL_BYTES", "0")
+    for dims, lv, op in [((1, 99999, 2), "w", "+"), ((1000001, 1, 2), "g", "max"), ((3, 4096, 2), "w", "*"),
+                         ((7, 513, 2), "gw", "&&"), ((2, 1000, 2), "w", "||"), ((123457, 1, 2), "g", "min")]:
+        x = recipes.make(KIND[op], dims, oracle.mask_of(lv), dtype, sum(dims))
+        init = recipes.make("ints", (oracle.out_count(dims, lv), 1, 1), 1, dtype, 8)
+        assert xr.xr_plan_describe(op, dtype, dims, lv, 256)["kernel"] == "colflat", (dims, lv)
+        check(op, dtype, dims, lv, gpu_reduce(op, dtype, dims, lv, x, init=init), x, init=init)
+        if dtype == "int32":
+            xb = recipes.make("bxor", dims, oracle.mask_of(lv), dtype, dims[1])
+            check("^", dtype, dims, lv, gpu_reduce("^", dtype, dims, lv, xb), xb)
