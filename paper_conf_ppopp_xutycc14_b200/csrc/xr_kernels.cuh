@@ -841,13 +841,13 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
   // 8-B rows (r02: two 32-bit columns): a 16-B vector holds two whole rows,
   // element q of every vector is column q % 2 -- one column group of VEC
   // lanes whose lanes fold into the K columns at the end
-  const bool sub16 = row_bytes < 16;
+  const bool sub16 = sizeof(T) == 4 && row_bytes < 16;  // (compiled out for 8-byte types)
   const int G = sub16 ? 1 : (int)(row_bytes >> 4);  // 16-B column groups per row (1..256)
   const int64_t rp4k = 4096 / row_bytes;           // whole rows per (<= 4 KiB) load round
   // vectors per round (r02: rows of any multiple of 16 B, not only powers of
   // two): a round is rp4k whole rows, so thread t < NV always meets column
   // group t % G; threads >= NV idle (<= 6 % of the CTA)
-  const int NV = (int)(rp4k * row_bytes / 16);
+  const int NV = sub16 ? kBlock : (int)(rp4k * G);  // (8-B rows: 512 rows = 256 vectors)
   const int64_t nblk = (a.R + rp4k - 1) / rp4k;    // 4 KiB row blocks per batch
   T* out = static_cast<T*>(a.out);
   Acc* partials = static_cast<Acc*>(a.partials);
@@ -855,7 +855,7 @@ __global__ void __launch_bounds__(kBlock, XR_SEG_MINB) colflat_kernel(const __gr
     const int64_t b = u / a.S, s = u - b * a.S;
     const int64_t r0 = min(split_lo(nblk, a.S, s) * rp4k, a.R), r1 = min(split_lo(nblk, a.S, s + 1) * rp4k, a.R);
     const U128* __restrict__ base = reinterpret_cast<const U128*>(static_cast<const T*>(a.in) + (b * a.R + r0) * a.K);
-    const int64_t nv = (r1 - r0) * row_bytes / 16;  // whole 16-B vectors of the unit
+    const int64_t nv = sub16 ? ((r1 - r0) >> 1) : (r1 - r0) * (row_bytes >> 4);  // whole 16-B vectors of the unit
     Acc acc[U][VEC];
 #pragma unroll
     for (int k = 0; k < U; ++k)
