@@ -1926,6 +1926,10 @@ __global__ void __launch_bounds__(kBlock) shortrow_kernel(const __grid_constant_
   constexpr int VEC = 16 / (int)sizeof(T);
   constexpr int NVC = CH / 16;                 // vectors per chunk
   constexpr int E = CH / (int)sizeof(T);       // elements per chunk
+  // the block's outputs are staged in shared memory and stored as 16-B
+  // vectors (r02bq: 8 scalar stores per thread, 32 B apart across a warp,
+  // bound 8-B rows at 28 % of DRAM peak)
+  __shared__ __align__(16) T so[kBlock * (E / 2)];
   const T* in = static_cast<const T*>(a.in);
   T* out = static_cast<T*>(a.out);
   const int L = (int)a.L;                      // elements per row (power of two, <= E)
@@ -1933,21 +1937,42 @@ __global__ void __launch_bounds__(kBlock) shortrow_kernel(const __grid_constant_
   const int64_t nchunks = a.O / rpt;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  for (int64_t c = t0; c < nchunks; c += stride) {
-    const U128* p = reinterpret_cast<const U128*>(in + c * E);
-    U128 x[NVC];
+  const bool vst = ((uintptr_t)out & 15u) == 0;
+  // staging pays only when a thread holds several rows (r02br: one row per
+  // thread -- a warp's outputs already contiguous -- was 7-16 % slower staged)
+  const bool stage = rpt >= 2;
+  for (int64_t cb = (int64_t)blockIdx.x * blockDim.x; cb < nchunks; cb += stride) {  // block-uniform
+    const int64_t c = cb + threadIdx.x;
+    if (c < nchunks) {
+      const U128* p = reinterpret_cast<const U128*>(in + c * E);
+      U128 x[NVC];
 #pragma unroll
-    for (int v = 0; v < NVC; ++v) x[v] = ld_stream(p + v);
-    Acc acc = O::identity();
+      for (int v = 0; v < NVC; ++v) x[v] = ld_stream(p + v);
+      Acc acc = O::identity();
 #pragma unroll
-    for (int e = 0; e < E; ++e) {
-      acc = O::combine(acc, O::lift(unpack<T>(x[e / VEC], e % VEC)));
-      if (((e + 1) & (L - 1)) == 0) {  // row e / L complete
-        const int64_t o = c * rpt + e / L;
-        out[o] = merge_init<OP, T>(acc, out, o, a.init_from_out);
-        acc = O::identity();
+      for (int e = 0; e < E; ++e) {
+        acc = O::combine(acc, O::lift(unpack<T>(x[e / VEC], e % VEC)));
+        if (((e + 1) & (L - 1)) == 0) {  // row e / L complete
+          const int64_t o = c * rpt + e / L;
+          const T r = merge_init<OP, T>(acc, out, o, a.init_from_out);
+          if (stage) so[threadIdx.x * rpt + e / L] = r;
+          else out[o] = r;
+          acc = O::identity();
+        }
       }
     }
+    if (!stage) continue;  // (block-uniform)
+    __syncthreads();
+    const int64_t nb = min((int64_t)blockDim.x, nchunks - cb) * rpt;  // outputs of this block round
+    T* ob = out + cb * rpt;                                              // 16-B aligned when out is
+    int64_t done = 0;
+    if (vst) {
+      for (int64_t i = threadIdx.x; i < nb / VEC; i += blockDim.x)
+        *reinterpret_cast<U128*>(ob + i * VEC) = *reinterpret_cast<const U128*>(so + i * VEC);
+      done = nb / VEC * VEC;
+    }
+    for (int64_t i = done + threadIdx.x; i < nb; i += blockDim.x) ob[i] = so[i];
+    __syncthreads();  // so is rewritten by the next round
   }
   // rows of the last partial chunk: one thread per row, in element order
   for (int64_t o = nchunks * rpt + t0; o < a.O; o += stride) {
